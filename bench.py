@@ -1,0 +1,395 @@
+#!/usr/bin/env python
+"""Benchmark of the batched scan hot path on B200 (one JSON line on rank 0).
+
+Metric (BASELINE.json): Gelem/s (and % of the HBM roofline) of int32/f32 scans at 1/2/4/8
+GPUs.  Workload at N=1 = configs[1]: G = 4096 problems of N = 2^14 elements; one STEP is
+the four scans that config names -- add-scan of int32 and of f32, inclusive and exclusive
+-- each over the whole 2^26-element batch (256 MiB in + 256 MiB out per scan, larger
+than the 126 MB L2, so no flush is needed between steps).  Under torchrun (--gpus N > 1)
+every rank scans its own G = 4096 problems (problems mode, Case 1 of PAPER.md:191-193, no
+collective on the data path): weak scaling, value = elements of all ranks / max-over-ranks
+time.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--no-extras] [--sweep]
+
+`--impl reference` times the CPU oracle (the only reference this paper-only run has) on
+host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+G_C2, N_C2 = 4096, 1 << 14
+SEED = 0x5CA2018
+METRIC = "Gelem/s and % of HBM roofline, int32/f32 scan at 1/2/4/8 B200"
+VARIANTS = [("i32", "add", "inclusive"), ("i32", "add", "exclusive"),
+            ("f32", "add", "inclusive"), ("f32", "add", "exclusive")]
+DIST = {"i32": "i32", "f32": "f32u"}
+TDT = {"i32": torch.int32, "f32": torch.float32}
+NPDT = {"i32": np.int32, "f32": np.float32}
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured", d
+    return 6650.0, "fallback (B200_PROFILING.md)", {}
+
+
+# ---------------------------------------------------------------- clocks during the timed region
+class ClockSampler:
+    def __init__(self, dev_index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8): "hw_slowdown",
+            getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40): "hw_thermal_slowdown",
+            getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20): "sw_thermal_slowdown",
+            getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4): "sw_power_cap",
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in names.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+# ---------------------------------------------------------------- the device workload
+def make_inputs(rank: int, device):
+    import inputs
+    xs = {}
+    for dt in ("i32", "f32"):
+        t = torch.empty(G_C2 * N_C2, dtype=torch.int32, device=device)
+        inputs.fill_device(t, DIST[dt], SEED + 2, offset=rank * G_C2 * N_C2)
+        xs[dt] = t.view(TDT[dt]).view(G_C2, N_C2)
+    return xs
+
+
+def step(sb, xs, outs, events=None):
+    for i, (dt, op, kind) in enumerate(VARIANTS):
+        if events is not None:
+            events[i][0].record()
+        sb.scan(xs[dt], op, kind, out=outs[i])
+        if events is not None:
+            events[i][1].record()
+
+
+def timed_steps(sb, xs, outs, K, per_launch=False):
+    """K steps between two events on the launching stream; optionally per-launch events."""
+    ev = None
+    if per_launch:
+        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in VARIANTS] for _ in range(K)]
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    s0.record()
+    for k in range(K):
+        step(sb, xs, outs, ev[k] if ev else None)
+    s1.record()
+    torch.cuda.synchronize()
+    total_ms = s0.elapsed_time(s1)
+    launch_ms = None
+    if ev:
+        launch_ms = [statistics.mean(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(K))
+                     for i in range(len(VARIANTS))]
+    return total_ms, launch_ms
+
+
+def e2e(sb, K=3):
+    """The same step through the public host-buffer API: pinned host in -> scan -> host out."""
+    import inputs
+    hin, hout = {}, []
+    for dt in ("i32", "f32"):
+        a = torch.empty(G_C2 * N_C2, dtype=torch.int32, pin_memory=True).numpy().view(NPDT[dt])
+        a[:] = inputs.generate(DIST[dt], G_C2 * N_C2, SEED + 2)
+        hin[dt] = a.reshape(G_C2, N_C2)
+    for _ in VARIANTS:
+        hout.append(torch.empty(G_C2 * N_C2, dtype=torch.int32, pin_memory=True).numpy()
+                    .view(np.int32).reshape(G_C2, N_C2))
+
+    def one():
+        for i, (dt, op, kind) in enumerate(VARIANTS):
+            sb.scan_host(hin[dt], op, kind, out=hout[i].view(NPDT[dt]))
+    one()
+    t0 = time.perf_counter()
+    for _ in range(K):
+        one()
+    dt_s = (time.perf_counter() - t0) / K
+    elems = len(VARIANTS) * G_C2 * N_C2
+    return {"value": elems / dt_s / 1e9, "unit": "Gelem/s", "ms_per_step": dt_s * 1e3, "steps": K,
+            "h2d_bytes_per_step": elems * 4, "d2h_bytes_per_step": elems * 4,
+            "api": "scan_batch_host (pinned host buffers, library-pipelined H2D/scan/D2H)"}
+
+
+# ---------------------------------------------------------------- CPU oracle (reference arm / baseline)
+def cpu_oracle_rate(budget_s: float = 12.0):
+    """The oracle as it stands (one thread, sequential C loop) on the same workload: it
+    scans whole 2^26-element variants of the c2 batch until the time budget is used."""
+    import inputs
+    import oracle
+    xs = {dt: inputs.generate(DIST[dt], G_C2 * N_C2, SEED + 2).reshape(G_C2, N_C2) for dt in ("i32", "f32")}
+    oracle.scan(xs["i32"][:4], "add")            # load / build
+    done, t_scan, steps = 0, 0.0, 0
+    while t_scan < budget_s or steps < 1:
+        for dt, op, kind in VARIANTS:
+            t0 = time.perf_counter()
+            oracle.scan(xs[dt], op, kind)
+            t_scan += time.perf_counter() - t0
+            done += G_C2 * N_C2
+        steps += 1
+    return {"value": done / t_scan / 1e9, "unit": "Gelem/s", "cores": 1, "kind": "oracle",
+            "sample": "%d full steps of the c2 workload (4 x 4096 x 2^14 elements each), "
+                      "single-threaded C oracle, %.1f s of scan time" % (steps, t_scan),
+            "host_cpu": _cpu_name(), "host_cores_available": len(os.sched_getaffinity(0)),
+            "ms_per_step": t_scan / steps * 1e3}
+
+
+def _cpu_name():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+# ---------------------------------------------------------------- extra configs (context)
+def extras(sb, dev):
+    import inputs
+    out = {}
+    # c1: N = 2^20, G = 1, inclusive int32 add: latency-bound, L2 resident
+    x = torch.empty(1 << 20, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "i32", SEED + 1)
+    y = torch.empty_like(x)
+    for _ in range(10):
+        sb.scan(x, "add", out=y)
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    s0.record()
+    for _ in range(200):
+        sb.scan(x, "add", out=y)
+    s1.record()
+    torch.cuda.synchronize()
+    us = s0.elapsed_time(s1) / 200 * 1e3
+    out["c1_i32_incl_N2^20"] = {"us_per_scan": us, "Gelem/s": (1 << 20) / us / 1e3,
+                                "note": "L2-resident (8 MiB), back-to-back launches"}
+    del x, y
+    # c3: N = 2^30 f32 inclusive add, single problem (look-back)
+    N = 1 << 30
+    x = torch.empty(N, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "f32u", SEED + 3)
+    x = x.view(torch.float32)
+    y = torch.empty_like(x)
+    for _ in range(3):
+        sb.scan(x, "add", out=y)
+    torch.cuda.synchronize()
+    s0.record()
+    for _ in range(10):
+        sb.scan(x, "add", out=y)
+    s1.record()
+    torch.cuda.synchronize()
+    ms = s0.elapsed_time(s1) / 10
+    hbm, _, _ = _peaks()
+    gbs = 8.0 * N / (ms * 1e-3) / 1e9
+    out["c3_f32_incl_N2^30"] = {"ms": ms, "Gelem/s": N / ms / 1e6, "GB/s": gbs,
+                                "frac_measured_hbm": gbs / hbm, "frac_8TBs": gbs / 8000.0}
+    del x, y
+    torch.cuda.empty_cache()
+    return out
+
+
+def sweep(sb, dev):
+    """On-box parameter search (the automated form of the paper's K search)."""
+    import inputs
+    rows = []
+    shapes = [(1, 1 << 20), (1, 1 << 24), (1, 1 << 28), (4096, 1 << 14), (1 << 16, 1 << 10),
+              (1 << 14, 1 << 12), (256, 1 << 20), (16, 1 << 24), (1 << 18, 1 << 8), (1 << 20, 1 << 6)]
+    cands = [("lookback", 0), ("lookback", 1), ("lookback", 2), ("cascade_cta", -1), ("cascade_warp", -1),
+             ("three_stage", 0)]
+    for G, N in shapes:
+        x = torch.empty(G * N, dtype=torch.int32, device=dev)
+        inputs.fill_device(x, "i32", 1)
+        x = x.view(G, N)
+        y = torch.empty_like(x)
+        for algo, param in cands:
+            if algo == "cascade_cta" and G < 148:
+                continue
+            if algo == "cascade_warp" and (G < 1024 or N > (1 << 16)):
+                continue
+            for _ in range(3):
+                sb.scan(x, "add", out=y, algo=algo, param=param)
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            reps = 20
+            torch.cuda.synchronize()
+            s0.record()
+            for _ in range(reps):
+                sb.scan(x, "add", out=y, algo=algo, param=param)
+            s1.record()
+            torch.cuda.synchronize()
+            ms = s0.elapsed_time(s1) / reps
+            rows.append({"G": G, "N": N, "algo": algo, "param": param, "ms": ms,
+                         "GB/s": 8.0 * G * N / ms / 1e6})
+            print(json.dumps(rows[-1]), file=sys.stderr, flush=True)
+        del x, y
+    return rows
+
+
+# ---------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--sweep", action="store_true")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    hbm, hbm_src, _ = _peaks()
+    config = {"workload": "configs[1]: batch scan G=4096 x N=2^14 per GPU, int32 and f32 add, "
+                          "inclusive and exclusive (4 scans per step)",
+              "G_per_gpu": G_C2, "N": N_C2, "layout": "row-major, stride N",
+              "l2": "inputs larger than L2 (256 MiB in + 256 MiB out per scan), no flush",
+              "parallelism": "problems sharded by rank (Case 1)" if world > 1 else "single GPU"}
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        r = cpu_oracle_rate()
+        print(json.dumps({"impl": "reference", "metric": METRIC, "value": r["value"], "unit": "Gelem/s",
+                          "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+                          "ms_per_step": r["ms_per_step"], "higher_is_better": True, "scaling": "weak",
+                          "vs_baseline": None, "dtype": "i32+f32", "data": "synthetic (splitmix64)",
+                          "config": config, "cpu_baseline": r,
+                          "e2e": {"value": r["value"], "unit": "Gelem/s", "h2d_bytes_per_step": 0,
+                                  "d2h_bytes_per_step": 0}}), flush=True)
+        return
+
+    import paper_conf_ipps_dieguezadnm18_b200 as sb
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    if args.sweep:
+        rows = sweep(sb, dev)
+        if rank == 0:
+            print(json.dumps({"sweep": rows}))
+        return
+
+    xs = make_inputs(rank, dev)
+    outs = [torch.empty((G_C2, N_C2), dtype=TDT[dt], device=dev) for dt, _, _ in VARIANTS]
+    for _ in range(max(args.warmup, 3)):
+        step(sb, xs, outs)
+    torch.cuda.synchronize()
+
+    # timed region: barrier + synchronize on both sides, device events, max over ranks
+    if world > 1:
+        torch.distributed.barrier()
+    with ClockSampler(local) as clk:
+        total_ms, _ = timed_steps(sb, xs, outs, args.steps)
+    if world > 1:
+        torch.distributed.barrier()
+        t = torch.tensor([total_ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        total_ms = float(t.item())
+    # per-launch durations (separate pass, same launches, events around each launch)
+    _, launch_ms = timed_steps(sb, xs, outs, max(10, args.steps // 10), per_launch=True)
+
+    ms_step = total_ms / args.steps
+    elems_step = len(VARIANTS) * G_C2 * N_C2 * world
+    value = elems_step / (ms_step * 1e-3) / 1e9
+    bytes_launch = 2 * 4 * G_C2 * N_C2
+    dom = max(range(len(VARIANTS)), key=lambda i: launch_ms[i])
+    achieved = bytes_launch / (launch_ms[dom] * 1e-3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    res = {
+        "metric": METRIC, "value": value, "unit": "Gelem/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "i32+f32", "data": "synthetic (splitmix64 counter-based, device-generated)",
+        "config": config,
+        "hbm_frac_of_step": {"algorithmic_GB/s": elems_step / world * 8 / (ms_step * 1e-3) / 1e9,
+                             "frac": elems_step / world * 8 / (ms_step * 1e-3) / 1e9 / hbm, "peak_src": hbm_src},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "traffic": traffic,
+                     "kernel": "lookback_kernel (%s %s %s), %d B algorithmic per launch" % (
+                         VARIANTS[dom] + (bytes_launch,)),
+                     "peak_src": hbm_src + " copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"},
+        "per_launch_ms": {"%s_%s_%s" % v: m for v, m in zip(VARIANTS, launch_ms)},
+        "gpu_launches": len(VARIANTS) * args.steps,
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and not args.no_e2e:
+        res["e2e"] = e2e(sb)
+    if rank == 0 and world == 1:
+        res["cpu_baseline"] = cpu_oracle_rate()
+    if rank == 0 and world == 1 and not args.no_extras:
+        del xs, outs
+        torch.cuda.empty_cache()
+        res["extras"] = extras(sb, dev)
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -64,6 +64,8 @@ def _load():
             lib.oracle_scan_add_f32.restype = None
             lib.oracle_total_add_u32.argtypes = [P, P, I, I]
             lib.oracle_total_add_f32.argtypes = [P, P, I, I]
+            lib.oracle_stream_add_u32.argtypes = [P, P, I, P, ctypes.c_int]
+            lib.oracle_stream_add_f32.argtypes = [P, P, P, I, P, P, ctypes.c_int]
             _lib = lib
     return _lib
 
@@ -145,3 +147,31 @@ def identity(op: str, dtype) -> float | int:
     if dtype == np.uint32:
         return 0
     return float("-inf")
+
+
+class StreamAdd:
+    """Streaming oracle for ONE long add-scan fed chunk by chunk (oracle_stream_add_*).
+
+    ``feed(chunk)`` returns the reference of that chunk (u32 bits for ints; fp64 prefix and
+    the |x| prefix for f32), continuing the running value from the previous chunk.
+    """
+
+    def __init__(self, dtype, kind: str = "inclusive"):
+        self.dtype = np.dtype(dtype)
+        self.excl = 1 if kind == "exclusive" else 0
+        self.acc_u = np.zeros(1, np.uint32)
+        self.acc_d = np.zeros(1, np.float64)
+        self.acc_a = np.zeros(1, np.float64)
+
+    def feed(self, x: np.ndarray):
+        x = np.ascontiguousarray(x)
+        lib = _load()
+        n = x.shape[0]
+        if self.dtype == np.float32:
+            y = np.empty(n, np.float64)
+            a = np.empty(n, np.float64)
+            lib.oracle_stream_add_f32(_ptr(x), _ptr(y), _ptr(a), n, _ptr(self.acc_d), _ptr(self.acc_a), self.excl)
+            return y, a
+        y = np.empty(n, np.uint32)
+        lib.oracle_stream_add_u32(_ptr(x), _ptr(y), n, _ptr(self.acc_u), self.excl)
+        return y.view(self.dtype)

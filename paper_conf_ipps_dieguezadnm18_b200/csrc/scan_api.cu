@@ -1,0 +1,440 @@
+// scan_api.cu -- the C-ABI of libscanb200.so (declared in include/scan_b200.h):
+// argument checks, workspace management, kernel selection, the host-buffer pipeline and
+// the sharded-mode steps.  Every computation is a launch of this library's kernels.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <tuple>
+#include <mutex>
+#include <utility>
+#include <vector>
+
+#include "scan_b200.h"
+#include "scan_internal.h"
+
+using namespace scanb200;
+
+namespace {
+
+constexpr size_t kCtlBytes = 256;          // [0] ticket [1] done [2] epoch (look-back)
+constexpr int kTargetCtas = 148 * 8;       // chunk count target of the three-stage path
+
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+bool valid_enums(scan_op op, scan_dtype dt, scan_kind kind) {
+    return (op == SCAN_OP_ADD || op == SCAN_OP_MAX) &&
+           (dt == SCAN_I32 || dt == SCAN_U32 || dt == SCAN_F32) &&
+           (kind == SCAN_INCLUSIVE || kind == SCAN_EXCLUSIVE);
+}
+
+OpCode opcode(scan_op op, scan_dtype dt) {
+    if (op == SCAN_OP_ADD) return dt == SCAN_F32 ? OpCode::AddF32 : OpCode::AddU32;
+    if (dt == SCAN_I32) return OpCode::MaxI32;
+    if (dt == SCAN_U32) return OpCode::MaxU32;
+    return OpCode::MaxF32;
+}
+
+bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == SCAN_F32; }
+
+// ---------------------------------------------------------------- dispatch
+// The analogue of the paper's empirical K search: the thresholds below come
+// from the on-box sweep recorded in profiles/ (bench.py --sweep).
+scan_algo choose_algo(int64_t N, int64_t G) {
+    (void)N; (void)G;
+    return SCAN_ALGO_LOOKBACK;
+}
+int choose_lookback_variant(int64_t N, int64_t G) {
+    int64_t total = N * G;
+    return total >= (int64_t(1) << 22) ? 1 : 0;
+}
+
+int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
+    const int64_t tile = chunk_tile_elems();
+    if (K > 0) return K * tile;
+    int64_t bx = std::max<int64_t>(1, (kTargetCtas + G - 1) / G);
+    int64_t chunk = (N + bx - 1) / bx;
+    chunk = std::max<int64_t>(tile, (chunk + tile - 1) / tile * tile);
+    return chunk;
+}
+
+// Look-back workspace: ctl | desc[C] (u64) | agg[C] (f64) | incl[C] (f64).  The layout
+// depends only on the workspace size (capacity C), never on the call, so a descriptor
+// slot is only ever read as a descriptor; packed and split modes share the u64 desc
+// array (split mode keeps tag|status in the low word and zero in the high word).
+constexpr size_t kLbSlotBytes = 24;
+size_t lookback_bytes(int64_t total, int variant, bool split) {
+    (void)split;
+    int64_t tile = lookback_tile_elems(variant);
+    int64_t tiles = (total + tile - 1) / tile;
+    return kCtlBytes + kLbSlotBytes * (size_t)tiles;
+}
+size_t three_stage_bytes(int64_t N, int64_t G, int64_t K) {
+    int64_t chunk = three_stage_chunk(N, G, K);
+    int64_t bx = (N + chunk - 1) / chunk;
+    return kCtlBytes + align_up(G * bx * 8, 256) + align_up(G * 8, 256);
+}
+
+// ---------------------------------------------------------------- workspace cache
+struct Ws { void* ptr = nullptr; size_t bytes = 0; };
+std::mutex g_ws_mu;
+// one cache per (device, stream, family): the look-back descriptors must never share
+// bytes with another family's scratch values
+enum Family { FAM_LOOKBACK = 0, FAM_CHUNKED = 1 };
+std::map<std::tuple<int, cudaStream_t, int>, Ws> g_ws;
+
+scan_status cached_workspace(cudaStream_t s, int fam, size_t need, void** out, size_t* out_bytes) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return SCAN_ERR_NO_DEVICE;
+    std::lock_guard<std::mutex> lk(g_ws_mu);
+    Ws& w = g_ws[std::make_tuple(dev, s, fam)];
+    if (w.bytes < need) {
+        size_t nb = std::max(need, w.bytes * 2);
+        if (w.ptr) cudaFreeAsync(w.ptr, s);
+        w.ptr = nullptr; w.bytes = 0;
+        if (cudaMallocAsync(&w.ptr, nb, s) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
+        if (cudaMemsetAsync(w.ptr, 0, nb, s) != cudaSuccess) return SCAN_ERR_CUDA;
+        w.bytes = nb;
+    }
+    *out = w.ptr;
+    *out_bytes = w.bytes;
+    return SCAN_OK;
+}
+
+scan_status resolve_ws(void* ws, size_t ws_bytes, size_t need, cudaStream_t s, int fam, void** out,
+                       size_t* out_bytes) {
+    if (ws) {
+        if (ws_bytes < need) return SCAN_ERR_NO_MEMORY;
+        if (((uintptr_t)ws) % 256) return SCAN_ERR_INVALID_ARG;
+        *out = ws;
+        *out_bytes = ws_bytes;
+        return SCAN_OK;
+    }
+    return cached_workspace(s, fam, need, out, out_bytes);
+}
+
+// ---------------------------------------------------------------- argument checks
+bool device_accessible(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return false; }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+scan_status check_buffers(const void* in, const void* out, int64_t total, bool check_device) {
+    if (!in || !out) return SCAN_ERR_INVALID_ARG;
+    if (((uintptr_t)in) % 4 || ((uintptr_t)out) % 4) return SCAN_ERR_INVALID_ARG;
+    uintptr_t a = (uintptr_t)in, b = (uintptr_t)out, n = (uintptr_t)total * 4;
+    if (a != b && a < b + n && b < a + n) return SCAN_ERR_INVALID_ARG;     // partial overlap
+    if (check_device && (!device_accessible(in) || !device_accessible(out))) return SCAN_ERR_INVALID_ARG;
+    return SCAN_OK;
+}
+
+scan_status check_shape(int64_t N, int64_t G, int64_t* total) {
+    if (N < 0 || G < 0) return SCAN_ERR_INVALID_ARG;
+    if (N > 0 && G > (int64_t(1) << 62) / N) return SCAN_ERR_INVALID_ARG;
+    *total = N * G;
+    return SCAN_OK;
+}
+
+scan_status from_cuda(cudaError_t e) { return e == cudaSuccess ? SCAN_OK : SCAN_ERR_CUDA; }
+
+// ---------------------------------------------------------------- kernel families
+scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
+                         scan_kind kind, int variant, void* ws, size_t ws_bytes, cudaStream_t s) {
+    const int64_t total = N * G;
+    const int64_t cap = (int64_t)((ws_bytes - kCtlBytes) / kLbSlotBytes);
+    LookbackParams p{};
+    p.in = in; p.out = out; p.N = N; p.total = total;
+    char* base = (char*)ws;
+    p.ctl = (uint32_t*)base;
+    p.desc = (uint64_t*)(base + kCtlBytes);
+    p.agg = (double*)(base + kCtlBytes + 8 * (size_t)cap);
+    p.incl = (double*)(base + kCtlBytes + 16 * (size_t)cap);
+    p.capacity = cap;
+    p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+    p.exclusive = kind == SCAN_EXCLUSIVE;
+    return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
+}
+
+ChunkParams chunk_params(const void* in, void* out, int64_t N, int64_t G, scan_kind kind) {
+    ChunkParams p{};
+    p.in = in; p.out = out; p.N = N; p.G = G;
+    p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0) && (N % 4 == 0);
+    p.exclusive = kind == SCAN_EXCLUSIVE;
+    return p;
+}
+
+scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
+                            scan_kind kind, int64_t K, void* ws, const uint64_t* carry_src,
+                            int carry_rows, cudaStream_t s, bool stages12, bool stage3,
+                            uint64_t* totals_out) {
+    ChunkParams p = chunk_params(in, out, N, G, kind);
+    p.chunk = three_stage_chunk(N, G, K);
+    p.Bx = (N + p.chunk - 1) / p.chunk;
+    char* base = (char*)ws + kCtlBytes;
+    p.aux = (uint64_t*)base;
+    p.totals = totals_out ? totals_out : (uint64_t*)(base + align_up(G * p.Bx * 8, 256));
+    p.carry_src = carry_src;
+    p.carry_rows = carry_rows;
+    const OpCode oc = opcode(op, dt);
+    if (stages12) {
+        cudaError_t e = launch_chunk_reduce(oc, p, s);
+        if (e != cudaSuccess) return SCAN_ERR_CUDA;
+        e = launch_aux_scan(oc, p, s);
+        if (e != cudaSuccess) return SCAN_ERR_CUDA;
+    }
+    if (stage3) return from_cuda(launch_chunk_scan(oc, p, s));
+    return SCAN_OK;
+}
+
+scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
+                     scan_kind kind, scan_algo algo, int64_t param, void* ws, size_t ws_bytes,
+                     cudaStream_t s) {
+    if (algo == SCAN_ALGO_AUTO) algo = choose_algo(N, G);
+    switch (algo) {
+    case SCAN_ALGO_LOOKBACK: {
+        int variant = (param >= 0 && param <= 2) ? (int)param : choose_lookback_variant(N, G);
+        void* w = nullptr;
+        size_t wb = 0;
+        scan_status st = resolve_ws(ws, ws_bytes, lookback_bytes(N * G, variant, split_desc(op, dt)), s,
+                                    FAM_LOOKBACK, &w, &wb);
+        if (st != SCAN_OK) return st;
+        return run_lookback(in, out, N, G, op, dt, kind, variant, w, wb, s);
+    }
+    case SCAN_ALGO_CASCADE_CTA: {
+        ChunkParams p = chunk_params(in, out, N, G, kind);
+        p.chunk = std::max<int64_t>(N, 1); p.Bx = 1;
+        return from_cuda(launch_chunk_scan(opcode(op, dt), p, s));
+    }
+    case SCAN_ALGO_CASCADE_WARP: {
+        ChunkParams p = chunk_params(in, out, N, G, kind);
+        p.chunk = std::max<int64_t>(N, 1); p.Bx = 1;
+        return from_cuda(launch_warp_cascade(opcode(op, dt), p, s));
+    }
+    case SCAN_ALGO_THREE_STAGE: {
+        void* w = nullptr;
+        size_t wb = 0;
+        scan_status st = resolve_ws(ws, ws_bytes, three_stage_bytes(N, G, param), s, FAM_CHUNKED, &w, &wb);
+        if (st != SCAN_OK) return st;
+        return run_three_stage(in, out, N, G, op, dt, kind, param, w, nullptr, 0, s, true, true, nullptr);
+    }
+    default:
+        return SCAN_ERR_UNSUPPORTED;
+    }
+}
+
+// ---------------------------------------------------------------- host-buffer pipeline
+// Three streams per device: copy-in, compute, copy-out; S staging slots of kPiece
+// elements rotate through them so the H2D copy of unit u+1, the scan of unit u and the
+// D2H copy of unit u-1 overlap (both copy engines busy: PCIe is full duplex).
+constexpr int kSlots = 3;
+constexpr int64_t kPiece = int64_t(1) << 24;      // 64 MiB of 32-bit elements per slot
+
+struct HostCtx {
+    bool init = false;
+    cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
+    void* slot[kSlots] = {};
+    cudaEvent_t ev_in[kSlots] = {}, ev_scan[kSlots] = {}, ev_out[kSlots] = {};
+    uint64_t* piece_totals = nullptr;
+    int64_t piece_cap = 0;
+};
+std::mutex g_host_mu;
+std::map<int, HostCtx> g_host;
+
+scan_status host_ctx(int dev, HostCtx** out) {
+    HostCtx& c = g_host[dev];
+    if (!c.init) {
+        if (cudaStreamCreateWithFlags(&c.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamCreateWithFlags(&c.comp, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamCreateWithFlags(&c.d2h, cudaStreamNonBlocking) != cudaSuccess)
+            return SCAN_ERR_CUDA;
+        for (int k = 0; k < kSlots; ++k) {
+            if (cudaMalloc(&c.slot[k], kPiece * 4) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
+            if (cudaEventCreateWithFlags(&c.ev_in[k], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&c.ev_scan[k], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&c.ev_out[k], cudaEventDisableTiming) != cudaSuccess)
+                return SCAN_ERR_CUDA;
+        }
+        c.init = true;
+    }
+    *out = &c;
+    return SCAN_OK;
+}
+
+scan_status host_pipeline(const void* in_host, void* out_host, int64_t N, int64_t G, scan_op op,
+                          scan_dtype dt, scan_kind kind) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return SCAN_ERR_NO_DEVICE;
+    std::lock_guard<std::mutex> lk(g_host_mu);
+    HostCtx* c = nullptr;
+    scan_status st = host_ctx(dev, &c);
+    if (st != SCAN_OK) return st;
+    const bool pieces = N > kPiece;
+    const int64_t npieces = pieces ? (N + kPiece - 1) / kPiece : 0;
+    if (pieces && c->piece_cap < npieces) {
+        if (c->piece_totals) cudaFree(c->piece_totals);
+        c->piece_totals = nullptr;
+        if (cudaMalloc(&c->piece_totals, npieces * 8) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
+        c->piece_cap = npieces;
+    }
+    const int64_t per_group = pieces ? 1 : std::max<int64_t>(1, kPiece / N);
+    const int64_t units = pieces ? G * npieces : (G + per_group - 1) / per_group;
+    const char* src = (const char*)in_host;
+    char* dst = (char*)out_host;
+    for (int64_t u = 0; u < units; ++u) {
+        const int k = (int)(u % kSlots);
+        int64_t off, n_elem, j = 0, ng;
+        if (pieces) {
+            const int64_t g = u / npieces;
+            j = u % npieces;
+            off = g * N + j * kPiece;
+            n_elem = std::min<int64_t>(kPiece, N - j * kPiece);
+            ng = 1;
+        } else {
+            const int64_t g0 = u * per_group;
+            ng = std::min<int64_t>(per_group, G - g0);
+            off = g0 * N;
+            n_elem = ng * N;
+        }
+        if (u >= kSlots && cudaStreamWaitEvent(c->h2d, c->ev_out[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (cudaMemcpyAsync(c->slot[k], src + off * 4, n_elem * 4, cudaMemcpyHostToDevice, c->h2d) != cudaSuccess)
+            return SCAN_ERR_CUDA;
+        if (cudaEventRecord(c->ev_in[k], c->h2d) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (cudaStreamWaitEvent(c->comp, c->ev_in[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (pieces) {
+            // piece j of a problem: three-stage scan whose carry folds the totals of pieces 0..j-1
+            void* w = nullptr; size_t wb = 0;
+            st = cached_workspace(c->comp, FAM_CHUNKED, three_stage_bytes(n_elem, 1, 0), &w, &wb);
+            if (st != SCAN_OK) return st;
+            st = run_three_stage(c->slot[k], c->slot[k], n_elem, 1, op, dt, kind, 0, w, c->piece_totals,
+                                 (int)j, c->comp, true, true, c->piece_totals + j);
+        } else {
+            st = run_algo(c->slot[k], c->slot[k], N, ng, op, dt, kind, SCAN_ALGO_AUTO, -1, nullptr, 0, c->comp);
+        }
+        if (st != SCAN_OK) return st;
+        if (cudaEventRecord(c->ev_scan[k], c->comp) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (cudaStreamWaitEvent(c->d2h, c->ev_scan[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (cudaMemcpyAsync(dst + off * 4, c->slot[k], n_elem * 4, cudaMemcpyDeviceToHost, c->d2h) != cudaSuccess)
+            return SCAN_ERR_CUDA;
+        if (cudaEventRecord(c->ev_out[k], c->d2h) != cudaSuccess) return SCAN_ERR_CUDA;
+    }
+    return from_cuda(cudaStreamSynchronize(c->d2h));
+}
+
+}  // namespace
+
+// =================================================================== exported C-ABI
+extern "C" {
+
+const char* scan_status_string(scan_status s) {
+    switch (s) {
+    case SCAN_OK: return "SCAN_OK";
+    case SCAN_ERR_INVALID_ARG: return "SCAN_ERR_INVALID_ARG";
+    case SCAN_ERR_UNSUPPORTED: return "SCAN_ERR_UNSUPPORTED";
+    case SCAN_ERR_CUDA: return "SCAN_ERR_CUDA";
+    case SCAN_ERR_NCCL: return "SCAN_ERR_NCCL";
+    case SCAN_ERR_NO_MEMORY: return "SCAN_ERR_NO_MEMORY";
+    case SCAN_ERR_NO_DEVICE: return "SCAN_ERR_NO_DEVICE";
+    }
+    return "SCAN_ERR_UNKNOWN";
+}
+
+int scan_abi_version(void) { return SCAN_B200_ABI_VERSION; }
+
+size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, scan_algo algo, int64_t param) {
+    if (N <= 0 || G <= 0) return kCtlBytes;
+    if (algo == SCAN_ALGO_AUTO) algo = choose_algo(N, G);
+    if (algo == SCAN_ALGO_LOOKBACK) {
+        int variant = (param >= 0 && param <= 2) ? (int)param : choose_lookback_variant(N, G);
+        return lookback_bytes(N * G, variant, split_desc(op, dtype));
+    }
+    if (algo == SCAN_ALGO_THREE_STAGE) return three_stage_bytes(N, G, param);
+    return kCtlBytes;
+}
+
+scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
+                          scan_kind kind, scan_algo algo, int64_t param, void* workspace,
+                          size_t workspace_bytes, void* stream) {
+    if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
+    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_THREE_STAGE) return SCAN_ERR_UNSUPPORTED;
+    int64_t total = 0;
+    scan_status st = check_shape(N, G, &total);
+    if (st != SCAN_OK) return st;
+    if (total == 0) return SCAN_OK;
+    st = check_buffers(in, out, total, true);
+    if (st != SCAN_OK) return st;
+    if (algo == SCAN_ALGO_THREE_STAGE && param < 0) return SCAN_ERR_INVALID_ARG;
+    return run_algo(in, out, N, G, op, dtype, kind, algo, param, workspace, workspace_bytes,
+                    (cudaStream_t)stream);
+}
+
+scan_status scan_batch(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
+                       scan_kind kind, void* stream) {
+    return scan_batch_ex(in, out, N, G, op, dtype, kind, SCAN_ALGO_AUTO, -1, nullptr, 0, stream);
+}
+
+scan_status scan_batch_host(const void* in_host, void* out_host, int64_t N, int64_t G, scan_op op,
+                            scan_dtype dtype, scan_kind kind) {
+    if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
+    int64_t total = 0;
+    scan_status st = check_shape(N, G, &total);
+    if (st != SCAN_OK) return st;
+    if (total == 0) return SCAN_OK;
+    st = check_buffers(in_host, out_host, total, false);
+    if (st != SCAN_OK) return st;
+    if (N > (int64_t(1) << 54)) return SCAN_ERR_UNSUPPORTED;      // piece count must fit an int
+    return host_pipeline(in_host, out_host, N, G, op, dtype, kind);
+}
+
+// ---------------------------------------------------------------- sharded problems
+size_t scan_shard_workspace_bytes(int64_t N_local, int64_t G) {
+    if (N_local <= 0 || G <= 0) return kCtlBytes;
+    return three_stage_bytes(N_local, G, 0);
+}
+
+scan_status scan_shard_totals(const void* in_local, int64_t N_local, int64_t G, scan_op op, scan_dtype dtype,
+                              void* totals_dev, void* workspace, size_t workspace_bytes, void* stream) {
+    if (!valid_enums(op, dtype, SCAN_INCLUSIVE)) return SCAN_ERR_INVALID_ARG;
+    int64_t total = 0;
+    scan_status st = check_shape(N_local, G, &total);
+    if (st != SCAN_OK) return st;
+    if (G == 0) return SCAN_OK;
+    if (!totals_dev || ((uintptr_t)totals_dev) % 8) return SCAN_ERR_INVALID_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (total > 0) {            // an empty portion still writes the identity totals (Stage 2 only)
+        st = check_buffers(in_local, in_local, total, true);
+        if (st != SCAN_OK) return st;
+    }
+    void* w = nullptr;
+    size_t wb = 0;
+    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_CHUNKED, &w, &wb);
+    if (st != SCAN_OK) return st;
+    return run_three_stage(in_local, nullptr, N_local, G, op, dtype, SCAN_INCLUSIVE, 0, w, nullptr, 0, s,
+                           true, false, (uint64_t*)totals_dev);
+}
+
+scan_status scan_shard_scan(const void* in_local, void* out_local, int64_t N_local, int64_t G, scan_op op,
+                            scan_dtype dtype, scan_kind kind, const void* all_totals_dev, int rank, int ngpu,
+                            void* workspace, size_t workspace_bytes, void* stream) {
+    if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
+    if (ngpu < 1 || rank < 0 || rank >= ngpu) return SCAN_ERR_INVALID_ARG;
+    int64_t total = 0;
+    scan_status st = check_shape(N_local, G, &total);
+    if (st != SCAN_OK) return st;
+    if (total == 0) return SCAN_OK;
+    if (rank > 0 && (!all_totals_dev || ((uintptr_t)all_totals_dev) % 8)) return SCAN_ERR_INVALID_ARG;
+    st = check_buffers(in_local, out_local, total, true);
+    if (st != SCAN_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    void* w = nullptr;
+    size_t wb = 0;
+    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_CHUNKED, &w, &wb);
+    if (st != SCAN_OK) return st;
+    return run_three_stage(in_local, out_local, N_local, G, op, dtype, kind, 0, w,
+                           (const uint64_t*)all_totals_dev, rank, s, false, true, nullptr);
+}
+
+}  // extern "C"

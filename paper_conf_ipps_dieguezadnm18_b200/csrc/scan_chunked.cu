@@ -1,0 +1,228 @@
+// scan_chunked.cu -- per-problem chunked kernels: the paper's cascade (PAPER.md:126 [§3.1,
+// Fig. 5]) and three-stage reduce-then-scan (PAPER.md:110-118 [§3.1, Fig. 3]), on sm_100a.
+//
+//   chunk_reduce  (Stage 1, "Chunk Reduce")      one CTA per (problem, chunk); the CTA walks
+//                                                the chunk tile by tile (cascade, K tiles)
+//                                                and writes one value per chunk to aux.
+//   aux_scan      (Stage 2, "Intermediate Scan") one WARP per problem (L_y^2 = warps per
+//                                                block problems per CTA);
+//                                                exclusive scan of the Bx chunk values in
+//                                                place + the problem total.
+//   chunk_scan    (Stage 3, "Scan+Addition")     one CTA per (problem, chunk); carry =
+//                                                (rank carry rows) . aux prefix, then a
+//                                                cascade over the chunk's tiles.  With one
+//                                                chunk per problem and no aux this is the
+//                                                CTA-per-problem batch kernel (L_y = 1).
+//   warp_cascade                                  one WARP per problem, cascade over
+//                                                V*128-element windows (small/medium N).
+//
+// Aux, totals and carry slots are 8 bytes: the 32-bit value in the low half, or the fp64
+// carry of f32 add.  All problem-local indices are 64-bit (N*G reaches 2^36).
+#include "scan_common.cuh"
+#include "scan_internal.h"
+
+namespace scanb200 {
+
+namespace {
+
+constexpr int CH_WARPS = 8, CH_V = 4;           // chunk kernels: 4096-element tiles
+constexpr int WC_WARPS = 8, WC_V = 8;           // warp cascade: 1024-element windows per warp
+
+template <class C> __device__ __forceinline__ C slot_get(uint64_t s);
+template <> __device__ __forceinline__ uint32_t slot_get<uint32_t>(uint64_t s) { return (uint32_t)s; }
+template <> __device__ __forceinline__ int32_t slot_get<int32_t>(uint64_t s) { return (int32_t)(uint32_t)s; }
+template <> __device__ __forceinline__ float slot_get<float>(uint64_t s) { return __uint_as_float((uint32_t)s); }
+template <> __device__ __forceinline__ double slot_get<double>(uint64_t s) { return __longlong_as_double((long long)s); }
+__device__ __forceinline__ uint64_t slot_put(uint32_t v) { return v; }
+__device__ __forceinline__ uint64_t slot_put(int32_t v) { return (uint32_t)v; }
+__device__ __forceinline__ uint64_t slot_put(float v) { return __float_as_uint(v); }
+__device__ __forceinline__ uint64_t slot_put(double v) { return (uint64_t)__double_as_longlong(v); }
+
+template <class C> __device__ __forceinline__ C shfl_up_c(C v, int d) {
+    if constexpr (sizeof(C) == 8) return __shfl_up_sync(FULL, v, d);
+    else return from_bits<C>(__shfl_up_sync(FULL, to_bits<C>(v), d));
+}
+template <class C> __device__ __forceinline__ C shfl_idx_c(C v, int s) {
+    if constexpr (sizeof(C) == 8) return __shfl_sync(FULL, v, s);
+    else return from_bits<C>(__shfl_sync(FULL, to_bits<C>(v), s));
+}
+
+// ------------------------------------------------------------------ Stage 1
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
+    __shared__ C s_part[WARPS];
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x / p.Bx, c = (int64_t)blockIdx.x % p.Bx;
+    const int64_t row = g * p.N;
+    const int64_t start = c * p.chunk;
+    const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
+    const T* in = (const T*)p.in;
+
+    C acc = Op::cidentity();
+    for (int64_t off = start + warp * WCH; off < end; off += TILE) {
+        Row4<T> x[V];
+#pragma unroll
+        for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, row + off + j * 128 + lane * 4, row + end, p.vec);
+        T t = Op::identity();
+#pragma unroll
+        for (int j = 0; j < V; ++j)
+#pragma unroll
+            for (int k = 0; k < 4; ++k) t = Op::apply(t, x[j].v[k]);
+        acc = Op::capply(acc, Op::to_carry(t));
+    }
+    acc = warp_reduce_carry<Op>(acc);
+    if (lane == 0) s_part[warp] = acc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        C tot = Op::cidentity();
+#pragma unroll
+        for (int w = 0; w < WARPS; ++w) tot = Op::capply(tot, s_part[w]);
+        p.aux[g * p.Bx + c] = slot_put(tot);
+    }
+}
+
+// ------------------------------------------------------------------ Stage 2
+template <class Op, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) aux_scan_kernel(ChunkParams p) {
+    using C = typename Op::Carry;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    if (g >= p.G) return;
+    uint64_t* a = p.aux + g * p.Bx;
+    C run = Op::cidentity();
+    for (int64_t b = 0; b < p.Bx; b += 32) {
+        const int64_t i = b + lane;
+        C v = i < p.Bx ? slot_get<C>(a[i]) : Op::cidentity();
+        C incl = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            C y = shfl_up_c<C>(incl, d);
+            if (lane >= d) incl = Op::capply(y, incl);
+        }
+        C ex = shfl_up_c<C>(incl, 1);
+        if (lane == 0) ex = Op::cidentity();
+        if (i < p.Bx) a[i] = slot_put(Op::capply(run, ex));
+        run = Op::capply(run, shfl_idx_c<C>(incl, 31));
+    }
+    if (lane == 0) p.totals[g] = slot_put(run);
+}
+
+// ------------------------------------------------------------------ Stage 3 / CTA cascade
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
+    __shared__ T s_wval[2][WARPS];
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x / p.Bx, c = (int64_t)blockIdx.x % p.Bx;
+    const int64_t row = g * p.N;
+    const int64_t start = c * p.chunk;
+    const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
+    const T* in = (const T*)p.in;
+    T* out = (T*)p.out;
+
+    // Stage 2 results folded in: carries of earlier ranks (sharded mode),
+    // then the exclusive prefix of the chunks before this one.
+    C carry = Op::cidentity();
+    for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * p.G + g]));
+    if (p.aux) carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
+
+    int it = 0;
+    for (int64_t off = start; off < end; off += TILE, ++it) {
+        WarpTile<Op, false, V> wt;
+        const int64_t wb = row + off + warp * WCH;
+        wt.load(in, wb, row + end, p.vec);
+        wt.scan();
+        if (lane == 0) s_wval[it & 1][warp] = wt.wtot;
+        __syncthreads();
+        T wp = Op::identity(), tot = Op::identity();
+#pragma unroll
+        for (int w = 0; w < WARPS; ++w) {
+            T v = s_wval[it & 1][w];
+            if (w < warp) wp = Op::apply(wp, v);
+            tot = Op::apply(tot, v);
+        }
+        wt.store(out, wb, row + end, p.vec, wp, false, Op::from_carry(carry), p.exclusive);
+        carry = Op::capply(carry, Op::to_carry(tot));       // the cascade carry (Fig. 5)
+    }
+}
+
+// ------------------------------------------------------------------ warp-per-problem cascade
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5;
+    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    if (g >= p.G) return;
+    const int64_t row = g * p.N;
+    const T* in = (const T*)p.in;
+    T* out = (T*)p.out;
+    C carry = Op::cidentity();
+    for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * p.G + g]));
+    for (int64_t off = 0; off < p.N; off += WCH) {
+        WarpTile<Op, false, V> wt;
+        wt.load(in, row + off, row + p.N, p.vec);
+        wt.scan();
+        wt.store(out, row + off, row + p.N, p.vec, Op::identity(), false, Op::from_carry(carry), p.exclusive);
+        carry = Op::capply(carry, Op::to_carry(wt.wtot));
+    }
+}
+
+template <class Op>
+cudaError_t reduce_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = p.G * p.Bx;
+    if (blocks == 0) return cudaSuccess;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    chunk_reduce_kernel<Op, CH_WARPS, CH_V><<<(unsigned)blocks, CH_WARPS * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+template <class Op>
+cudaError_t auxscan_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = (p.G + 7) / 8;
+    if (blocks == 0) return cudaSuccess;
+    aux_scan_kernel<Op, 8><<<(unsigned)blocks, 8 * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+template <class Op>
+cudaError_t scan_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = p.G * p.Bx;
+    if (blocks == 0) return cudaSuccess;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    chunk_scan_kernel<Op, CH_WARPS, CH_V><<<(unsigned)blocks, CH_WARPS * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+template <class Op>
+cudaError_t warp_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = (p.G + WC_WARPS - 1) / WC_WARPS;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    warp_cascade_kernel<Op, WC_WARPS, WC_V><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
+#define SCANB200_DISPATCH(fn)                                          \
+    switch (op) {                                                      \
+    case OpCode::AddU32: return fn<OpAddU32>(p, s);                    \
+    case OpCode::MaxI32: return fn<OpMaxI32>(p, s);                    \
+    case OpCode::MaxU32: return fn<OpMaxU32>(p, s);                    \
+    case OpCode::MaxF32: return fn<OpMaxF32>(p, s);                    \
+    case OpCode::AddF32: return fn<OpAddF32>(p, s);                    \
+    }                                                                  \
+    return cudaErrorInvalidValue;
+
+}  // namespace
+
+int64_t chunk_tile_elems() { return CH_WARPS * 32 * CH_V * 4; }
+int64_t warp_tile_elems() { return WC_V * 128; }
+
+cudaError_t launch_chunk_reduce(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(reduce_op) }
+cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(auxscan_op) }
+cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(scan_op) }
+cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_op) }
+
+}  // namespace scanb200

@@ -1,0 +1,58 @@
+// scan_internal.h -- host-side interface between the C-ABI (scan_api.cu) and the kernels.
+// Not installed, not part of the public boundary (include/scan_b200.h is).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace scanb200 {
+
+enum class OpCode : int { AddU32 = 0, MaxI32 = 1, MaxU32 = 2, MaxF32 = 3, AddF32 = 4 };
+
+// ---------------------------------------------------------------- single-pass look-back
+struct LookbackParams {
+    const void* in;
+    void* out;
+    int64_t N;          // elements per problem (> 0)
+    int64_t total;      // G * N
+    uint32_t* ctl;      // [0] ticket, [1] done, [2] epoch   (zero-initialised once)
+    uint64_t* desc;     // descriptors: packed value<<32|tag<<2|status, or (f32 add) tag<<2|status
+    double* agg;        //   f32 add: tile aggregates (fp64)
+    double* incl;       //   f32 add: tile inclusive prefixes (fp64)
+    int64_t capacity;   // descriptor slots of the workspace (>= tiles of any call)
+    bool vec;           // in and out are 16-byte aligned
+    bool exclusive;
+};
+int64_t lookback_tile_elems(int variant);
+cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s);
+
+// ---------------------------------------------------------------- cascade / three-stage
+// Chunked per-problem kernels.  Problem g is cut into Bx chunks of `chunk` elements
+// (chunk = K * tile, the paper's cascade depth K).
+struct ChunkParams {
+    const void* in;
+    void* out;
+    int64_t N;              // elements per problem (local shard length in sharded mode)
+    int64_t G;
+    int64_t chunk;          // elements per chunk (multiple of the tile)
+    int64_t Bx;             // chunks per problem
+    uint64_t* aux;          // [G][Bx] 8-byte slots: chunk reductions, then exclusive prefixes
+    uint64_t* totals;       // [G] problem totals (Stage 2 output)
+    const uint64_t* carry_src;  // [carry_rows][G] slots folded into every problem's carry
+    int carry_rows;
+    bool vec;
+    bool exclusive;
+};
+int64_t chunk_tile_elems();
+int64_t warp_tile_elems();
+// Stage 1: aux[g][c] = reduction of chunk c of problem g
+cudaError_t launch_chunk_reduce(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Stage 2: exclusive scan of aux[g][*] in place, totals[g] = full reduction (L_y > 1
+// problems per block)
+cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Stage 3: scan of every chunk + carry (carry_src rows, then aux prefix when aux != null).
+// With Bx == 1 and aux == null this is the CTA-per-problem cascade.
+cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Warp-per-problem cascade (L_y = warps per block problems per CTA).
+cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s);
+
+}  // namespace scanb200

@@ -232,3 +232,17 @@ def test_degenerate_shapes():
     x = inputs.generate("i32", 10, 1).reshape(10, 1)         # N = 1: inclusive = x, exclusive = identity
     assert np.array_equal(oracle.scan(x, "add"), x)
     assert np.all(oracle.scan(x, "max", "exclusive") == -(2**31))
+
+
+@pytest.mark.parametrize("dist,kind", [("i32", "inclusive"), ("u32", "exclusive"), ("f32u", "inclusive"),
+                                       ("f32s", "exclusive")])
+def test_streaming_oracle_equals_one_shot(dist, kind):
+    x = inputs.generate(dist, 50000, 31)
+    s = oracle.StreamAdd(x.dtype, kind)
+    parts = [s.feed(x[a:b]) for a, b in [(0, 1), (1, 4097), (4097, 4097), (4097, 50000)]]
+    if x.dtype == np.float32:
+        ref, sabs = oracle.scan(x, "add", kind, with_abs=True)
+        assert np.array_equal(np.concatenate([p[0] for p in parts]), ref)
+        assert np.array_equal(np.concatenate([p[1] for p in parts]), sabs)
+    else:
+        assert np.array_equal(np.concatenate(parts), oracle.scan(x, "add", kind))
