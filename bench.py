@@ -250,36 +250,52 @@ def sweep(sb, dev):
     """On-box parameter search (the automated form of the paper's K search)."""
     import inputs
     rows = []
-    shapes = [(1, 1 << 20), (1, 1 << 24), (1, 1 << 28), (4096, 1 << 14), (1 << 16, 1 << 10),
-              (1 << 14, 1 << 12), (256, 1 << 20), (16, 1 << 24), (1 << 18, 1 << 8), (1 << 20, 1 << 6)]
-    cands = [("lookback", 0), ("lookback", 1), ("lookback", 2), ("cascade_cta", -1), ("cascade_warp", -1),
-             ("three_stage", 0)]
-    for G, N in shapes:
+    shapes = [("i32", 1, 1 << 20), ("i32", 1, 1 << 24), ("i32", 1, 1 << 28), ("f32", 1, 1 << 30),
+              ("i32", 4096, 1 << 14), ("f32", 4096, 1 << 14), ("i32", 1 << 16, 1 << 10),
+              ("i32", 1 << 14, 1 << 12), ("i32", 256, 1 << 20), ("i32", 16, 1 << 24), ("i32", 1 << 18, 1 << 8),
+              ("i32", 1 << 20, 1 << 6), ("i32", 1 << 13, 1 << 16)]
+    cands = [("lookback", v) for v in range(sb._lib.lib_num_lookback_variants())] + [
+        ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0)]
+    s = torch.cuda.Stream(dev)
+    for dt, G, N in shapes:
         x = torch.empty(G * N, dtype=torch.int32, device=dev)
-        inputs.fill_device(x, "i32", 1)
-        x = x.view(G, N)
+        inputs.fill_device(x, DIST[dt], 1)
+        x = x.view(TDT[dt]).view(G, N)
         y = torch.empty_like(x)
         for algo, param in cands:
             if algo == "cascade_cta" and G < 148:
                 continue
             if algo == "cascade_warp" and (G < 1024 or N > (1 << 16)):
                 continue
-            for _ in range(3):
-                sb.scan(x, "add", out=y, algo=algo, param=param)
-            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            reps = 20
-            torch.cuda.synchronize()
-            s0.record()
-            for _ in range(reps):
-                sb.scan(x, "add", out=y, algo=algo, param=param)
-            s1.record()
-            torch.cuda.synchronize()
-            ms = s0.elapsed_time(s1) / reps
-            rows.append({"G": G, "N": N, "algo": algo, "param": param, "ms": ms,
+            reps = 20 if G * N < (1 << 26) else 5
+            ms = device_time(lambda: sb.scan(x, "add", out=y, algo=algo, param=param, stream=s), s, reps)
+            rows.append({"dtype": dt, "G": G, "N": N, "algo": algo, "param": param, "ms": ms,
                          "GB/s": 8.0 * G * N / ms / 1e6})
             print(json.dumps(rows[-1]), file=sys.stderr, flush=True)
         del x, y
+        torch.cuda.empty_cache()
     return rows
+
+
+def device_time(fn, s, reps):
+    """Device time per call: warm up on stream s, capture `reps` calls into a CUDA graph,
+    replay it between two events (removes the Python/launch overhead from small cases)."""
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            fn()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(reps):
+            fn()
+    with torch.cuda.stream(s):
+        g.replay()
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(s)
+        g.replay()
+        s1.record(s)
+    torch.cuda.synchronize()
+    return s0.elapsed_time(s1) / reps
 
 
 # ---------------------------------------------------------------- main

@@ -22,7 +22,7 @@ STATUS = {0: "SCAN_OK", 1: "SCAN_ERR_INVALID_ARG", 2: "SCAN_ERR_UNSUPPORTED", 3:
 # every symbol include/scan_b200.h declares (checked by tests/test_abi.py)
 EXPORTS = ("scan_status_string", "scan_abi_version", "scan_batch", "scan_workspace_bytes",
            "scan_batch_ex", "scan_batch_host", "scan_shard_totals", "scan_shard_scan",
-           "scan_shard_workspace_bytes")
+           "scan_shard_workspace_bytes", "scan_debug_trace")
 
 
 class ScanError(RuntimeError):
@@ -47,6 +47,7 @@ def _load() -> ctypes.CDLL:
         "scan_shard_totals": ([P, I64, I64, I, I, P, P, SZ, P], I),
         "scan_shard_scan": ([P, P, I64, I64, I, I, I, P, I, I, P, SZ, P], I),
         "scan_shard_workspace_bytes": ([I64, I64], SZ),
+        "scan_debug_trace": ([P, I64], I),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -56,6 +57,10 @@ def _load() -> ctypes.CDLL:
 
 
 lib = _load()
+
+
+def lib_num_lookback_variants() -> int:
+    return 4
 
 
 def check(fn: str, code: int) -> None:

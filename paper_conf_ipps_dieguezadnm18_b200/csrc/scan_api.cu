@@ -43,13 +43,23 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 // ---------------------------------------------------------------- dispatch
 // The analogue of the paper's empirical K search: the thresholds below come
 // from the on-box sweep recorded in profiles/ (bench.py --sweep).
-scan_algo choose_algo(int64_t N, int64_t G) {
-    (void)N; (void)G;
+//   many problems of moderate N (rows 16-byte aligned): the paper's own batch mapping wins
+//     on B200 -- one CTA per problem (cascade, L_y = 1) for N >= 4096, one warp per problem
+//     (L_y = 8) for 1024 <= N < 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
+//   short rows (N < 1024) or unaligned rows: flat segmented look-back, one tile per CTA;
+//   few large problems (G*N >= 2^22): pipelined look-back with 64 KiB tiles;
+//   small totals (latency bound, L2 resident): pipelined look-back with 32 KiB tiles.
+// `aligned` = both base pointers 16-byte aligned.
+scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
+    const bool rows_aligned = aligned && (N % 4 == 0);
+    if (rows_aligned && G >= 592 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
+    if (rows_aligned && G >= 1184 && N >= 1024) return SCAN_ALGO_CASCADE_WARP;
     return SCAN_ALGO_LOOKBACK;
 }
 int choose_lookback_variant(int64_t N, int64_t G) {
-    int64_t total = N * G;
-    return total >= (int64_t(1) << 22) ? 1 : 0;
+    const int64_t total = N * G;
+    if (N < 1024 && G > 1) return 3;
+    return total >= (int64_t(1) << 22) ? 0 : 1;
 }
 
 int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
@@ -61,11 +71,11 @@ int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
     return chunk;
 }
 
-// Look-back workspace: ctl | desc[C] (u64) | agg[C] (f64) | incl[C] (f64).  The layout
-// depends only on the workspace size (capacity C), never on the call, so a descriptor
-// slot is only ever read as a descriptor; packed and split modes share the u64 desc
-// array (split mode keeps tag|status in the low word and zero in the high word).
-constexpr size_t kLbSlotBytes = 24;
+// Look-back workspace: ctl | desc[C] (16-byte slots).  The layout depends only on the
+// workspace size (capacity C), never on the call; every descriptor word carries the tag
+// of the launch that wrote it, so 8-byte (32-bit carries) and 16-byte (fp64 carries)
+// uses of the same bytes can never be confused.
+constexpr size_t kLbSlotBytes = 16;
 size_t lookback_bytes(int64_t total, int variant, bool split) {
     (void)split;
     int64_t tile = lookback_tile_elems(variant);
@@ -116,6 +126,10 @@ scan_status resolve_ws(void* ws, size_t ws_bytes, size_t need, cudaStream_t s, i
     return cached_workspace(s, fam, need, out, out_bytes);
 }
 
+// debug timeline buffer for the look-back kernels (scan_debug_trace)
+uint64_t* g_trace = nullptr;
+int64_t g_trace_tiles = 0;
+
 // ---------------------------------------------------------------- argument checks
 bool device_accessible(const void* p) {
     cudaPointerAttributes a;
@@ -151,9 +165,9 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     char* base = (char*)ws;
     p.ctl = (uint32_t*)base;
     p.desc = (uint64_t*)(base + kCtlBytes);
-    p.agg = (double*)(base + kCtlBytes + 8 * (size_t)cap);
-    p.incl = (double*)(base + kCtlBytes + 16 * (size_t)cap);
     p.capacity = cap;
+    p.trace = g_trace;
+    p.trace_tiles = g_trace_tiles;
     p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
     p.exclusive = kind == SCAN_EXCLUSIVE;
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
@@ -193,10 +207,13 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
 scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
                      scan_kind kind, scan_algo algo, int64_t param, void* ws, size_t ws_bytes,
                      cudaStream_t s) {
-    if (algo == SCAN_ALGO_AUTO) algo = choose_algo(N, G);
+    if (algo == SCAN_ALGO_AUTO) {
+        algo = choose_algo(N, G, (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0));
+        param = -1;
+    }
     switch (algo) {
     case SCAN_ALGO_LOOKBACK: {
-        int variant = (param >= 0 && param <= 2) ? (int)param : choose_lookback_variant(N, G);
+        int variant = (param >= 0 && param < lookback_num_variants()) ? (int)param : choose_lookback_variant(N, G);
         void* w = nullptr;
         size_t wb = 0;
         scan_status st = resolve_ws(ws, ws_bytes, lookback_bytes(N * G, variant, split_desc(op, dt)), s,
@@ -344,11 +361,22 @@ const char* scan_status_string(scan_status s) {
 
 int scan_abi_version(void) { return SCAN_B200_ABI_VERSION; }
 
+scan_status scan_debug_trace(void* device_buf, int64_t tiles) {
+    if (tiles < 0 || (tiles > 0 && !device_buf)) return SCAN_ERR_INVALID_ARG;
+    g_trace = tiles ? (uint64_t*)device_buf : nullptr;
+    g_trace_tiles = tiles;
+    return SCAN_OK;
+}
+
 size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, scan_algo algo, int64_t param) {
     if (N <= 0 || G <= 0) return kCtlBytes;
-    if (algo == SCAN_ALGO_AUTO) algo = choose_algo(N, G);
+    if (algo == SCAN_ALGO_AUTO) {
+        // pointer alignment is unknown here: cover the look-back choice (the only one that
+        // needs workspace) with its largest descriptor array (8192-element tiles)
+        return lookback_bytes(N * G, 1, split_desc(op, dtype));
+    }
     if (algo == SCAN_ALGO_LOOKBACK) {
-        int variant = (param >= 0 && param <= 2) ? (int)param : choose_lookback_variant(N, G);
+        int variant = (param >= 0 && param < lookback_num_variants()) ? (int)param : choose_lookback_variant(N, G);
         return lookback_bytes(N * G, variant, split_desc(op, dtype));
     }
     if (algo == SCAN_ALGO_THREE_STAGE) return three_stage_bytes(N, G, param);
@@ -366,7 +394,7 @@ scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_
     if (total == 0) return SCAN_OK;
     st = check_buffers(in, out, total, true);
     if (st != SCAN_OK) return st;
-    if (algo == SCAN_ALGO_THREE_STAGE && param < 0) return SCAN_ERR_INVALID_ARG;
+    if (algo == SCAN_ALGO_THREE_STAGE && param < 0) param = 0;          // auto K
     return run_algo(in, out, N, G, op, dtype, kind, algo, param, workspace, workspace_bytes,
                     (cudaStream_t)stream);
 }
@@ -391,8 +419,8 @@ scan_status scan_batch_host(const void* in_host, void* out_host, int64_t N, int6
 
 // ---------------------------------------------------------------- sharded problems
 size_t scan_shard_workspace_bytes(int64_t N_local, int64_t G) {
-    if (N_local <= 0 || G <= 0) return kCtlBytes;
-    return three_stage_bytes(N_local, G, 0);
+    if (N_local < 0 || G <= 0) return kCtlBytes;
+    return three_stage_bytes(N_local, G, 0);      // an empty portion still needs its G totals
 }
 
 scan_status scan_shard_totals(const void* in_local, int64_t N_local, int64_t G, scan_op op, scan_dtype dtype,

@@ -366,3 +366,189 @@ struct WarpTile {
 };
 
 }  // namespace scanb200
+
+namespace scanb200 {
+
+// ------------------------------------------------------------------ TMA bulk copies (sm_90+/sm_100a)
+// 1-D bulk copies global -> shared (SASS UBLKCP) completing on an mbarrier (SYNCS.*).  They
+// keep the bytes in flight without holding registers, so the number of outstanding loads
+// per SM is bounded by shared memory instead of the register file.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void tma_load_1d(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar,
+                                            uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+        :: "r"(smem_u32(dst_smem)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+}
+__device__ __forceinline__ uint64_t l2_evict_last_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+    asm volatile(
+        "{\n .reg .pred p;\n WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(phase) : "memory");
+}
+__device__ __forceinline__ uint4 lds_v4(const void* p) {
+    uint4 r;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "r"(smem_u32(p)));
+    return r;
+}
+
+// ------------------------------------------------------------------ the warp tile engine, smem-staged
+// Same row structure as WarpTile, but the rows live in shared memory (landed there by a
+// bulk copy) and are read twice: pass 1 computes the lane / row / warp prefixes (only
+// 2V values + 3 bitmasks stay in registers), pass 2 re-reads each row once the carry is
+// known and writes the outputs with 128-bit streaming stores.  Row reads are 512
+// contiguous bytes per warp instruction: bank-conflict free.
+template <class Op, bool SEG, int V>
+struct WarpTileS {
+    using T = typename Op::T;
+    static_assert(V <= 8, "head masks pack 4 bits per row into 32 bits");
+    T lin[V];
+    T rp[V];
+    uint32_t hdm = 0;     // 4 head bits per row
+    uint32_t lflm = 0;    // bit j: a head lies in lanes < lane of row j
+    uint32_t rpfm = 0;    // bit j: a head lies in rows < j of this warp
+    T wtot; bool wfl;
+
+    __device__ __forceinline__ void pass1(const T* srow, int o0, bool small, uint32_t r_tile, uint32_t N32,
+                                          int first) {
+        const int lane = lane_id();
+        T run = Op::identity(); bool f = false;
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+            unsigned hd = 0u;
+            if (SEG) {
+                int o = o0 + j * 128 + lane * 4;
+                hd = small ? row_heads_small((uint32_t)o, r_tile, N32) : row_heads_big(o, first);
+                hdm |= hd << (4 * j);
+            }
+            T v = row_reduce<Op, SEG>(x, hd);
+            unsigned hm = SEG ? __ballot_sync(FULL, hd != 0u) : 0u;
+            bool lf;
+            T incl = warp_seg_scan<Op, SEG>(v, hm, lin[j], lf);
+            if (SEG && lf) lflm |= 1u << j;
+            T rt = shfl_idx<T>(incl, 31);
+            rp[j] = run;
+            if (SEG && f) rpfm |= 1u << j;
+            run = SEG ? seg_fold<Op>(run, hm != 0u, rt) : Op::apply(run, rt);
+            f = f || (hm != 0u);
+        }
+        wtot = run; wfl = f;
+    }
+    // gout = output address of the warp's first element (global index gidx); `fast` = whole
+    // window in range and 16-byte aligned, else guarded stores against `limit`
+    __device__ __forceinline__ void pass2(const T* srow, T* out, int64_t gidx, int64_t limit, bool fast,
+                                          bool vec, bool excl_kind, T wp, bool wpf, T cin) {
+        const int lane = lane_id();
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+            T in; bool inf;
+            if (SEG) {
+                bool rf = (rpfm >> j) & 1u, lf = (lflm >> j) & 1u;
+                in = seg_fold<Op>(wp, rf, rp[j]); inf = wpf || rf;
+                in = seg_fold<Op>(in, lf, lin[j]); inf = inf || lf;
+            } else {
+                in = Op::apply(Op::apply(wp, rp[j]), lin[j]); inf = false;
+            }
+            unsigned hd = SEG ? (hdm >> (4 * j)) & 0xFu : 0u;
+            Row4<T> o = excl_kind ? row_output<Op, SEG, true>(x, hd, in, inf, cin)
+                                  : row_output<Op, SEG, false>(x, hd, in, inf, cin);
+            const int64_t idx = gidx + j * 128 + lane * 4;
+            if (fast) st_stream_v4(out + idx, row_to_u4<T>(o));
+            else store_row<Op>(out, idx, limit, vec, o);
+        }
+    }
+};
+
+// The same engine with the segmentation chosen per call (SEG is a per-tile runtime property
+// in the pipelined kernel, which keeps the state of two tiles in flight per warp).
+template <class Op, int V>
+struct WarpTileP {
+    using T = typename Op::T;
+    static_assert(V <= 8, "head masks pack 4 bits per row into 32 bits");
+    T lin[V];
+    T rp[V];
+    uint32_t hdm, lflm, rpfm;
+    T wtot; bool wfl;
+
+    template <bool SEG>
+    __device__ __forceinline__ void pass1(const T* srow, int o0, bool small, uint32_t r_tile, uint32_t N32,
+                                          int first) {
+        const int lane = lane_id();
+        hdm = 0u; lflm = 0u; rpfm = 0u;
+        T run = Op::identity(); bool f = false;
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+            unsigned hd = 0u;
+            if (SEG) {
+                int o = o0 + j * 128 + lane * 4;
+                hd = small ? row_heads_small((uint32_t)o, r_tile, N32) : row_heads_big(o, first);
+                hdm |= hd << (4 * j);
+            }
+            T v = row_reduce<Op, SEG>(x, hd);
+            unsigned hm = SEG ? __ballot_sync(FULL, hd != 0u) : 0u;
+            bool lf;
+            T incl = warp_seg_scan<Op, SEG>(v, hm, lin[j], lf);
+            if (SEG && lf) lflm |= 1u << j;
+            T rt = shfl_idx<T>(incl, 31);
+            rp[j] = run;
+            if (SEG && f) rpfm |= 1u << j;
+            run = SEG ? seg_fold<Op>(run, hm != 0u, rt) : Op::apply(run, rt);
+            f = f || (hm != 0u);
+        }
+        wtot = run; wfl = f;
+    }
+    template <bool SEG>
+    __device__ __forceinline__ void pass2(const T* srow, T* out, int64_t gidx, int64_t limit, bool fast,
+                                          bool vec, bool excl_kind, T wp, bool wpf, T cin) const {
+        const int lane = lane_id();
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+            T in; bool inf;
+            if (SEG) {
+                bool rf = (rpfm >> j) & 1u, lf = (lflm >> j) & 1u;
+                in = seg_fold<Op>(wp, rf, rp[j]); inf = wpf || rf;
+                in = seg_fold<Op>(in, lf, lin[j]); inf = inf || lf;
+            } else {
+                in = Op::apply(Op::apply(wp, rp[j]), lin[j]); inf = false;
+            }
+            unsigned hd = SEG ? (hdm >> (4 * j)) & 0xFu : 0u;
+            Row4<T> o = excl_kind ? row_output<Op, SEG, true>(x, hd, in, inf, cin)
+                                  : row_output<Op, SEG, false>(x, hd, in, inf, cin);
+            const int64_t idx = gidx + j * 128 + lane * 4;
+            if (fast) st_stream_v4(out + idx, row_to_u4<T>(o));
+            else store_row<Op>(out, idx, limit, vec, o);
+        }
+    }
+};
+
+}  // namespace scanb200

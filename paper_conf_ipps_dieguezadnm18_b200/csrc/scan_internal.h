@@ -15,14 +15,15 @@ struct LookbackParams {
     int64_t N;          // elements per problem (> 0)
     int64_t total;      // G * N
     uint32_t* ctl;      // [0] ticket, [1] done, [2] epoch   (zero-initialised once)
-    uint64_t* desc;     // descriptors: packed value<<32|tag<<2|status, or (f32 add) tag<<2|status
-    double* agg;        //   f32 add: tile aggregates (fp64)
-    double* incl;       //   f32 add: tile inclusive prefixes (fp64)
-    int64_t capacity;   // descriptor slots of the workspace (>= tiles of any call)
+    uint64_t* desc;     // descriptors: value<<32|tag<<2|status (two such words per tile for fp64)
+    int64_t capacity;   // 16-byte descriptor slots of the workspace (>= tiles of any call)
+    uint64_t* trace;    // debug: 4 %globaltimer stamps per tile (NULL in normal use)
+    int64_t trace_tiles;
     bool vec;           // in and out are 16-byte aligned
     bool exclusive;
 };
 int64_t lookback_tile_elems(int variant);
+int lookback_num_variants();
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s);
 
 // ---------------------------------------------------------------- cascade / three-stage

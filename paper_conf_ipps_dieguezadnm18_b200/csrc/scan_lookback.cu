@@ -4,24 +4,38 @@
 // Scan+Addition, PAPER.md:110-118 [§3.1, Fig. 3]), i.e. 3N element transfers, and notes
 // that its Stage 2 leaves the GPU "underused" at G=1.  On one B200 the
 // byte-optimal schedule is single pass (2N transfers): each tile publishes its aggregate
-// as soon as it has it and looks back over its predecessors' published values, the
+// as soon as it has it and looks back over its predecessors' published values -- the
 // barrier-free idea of StreamScan [25] that the paper cites.  The
-// three-stage form is kept in scan_three_stage.cu (deterministic mode + sharded path).
+// three-stage form is kept in scan_chunked.cu (deterministic mode + sharded path).
 //
 // The G problems of N elements are scanned as ONE flat array of G*N elements
-// cut into tiles of WARPS*32*V*4 elements; a tile that contains a problem start publishes
-// its (trailing-segment) inclusive value immediately, so every look-back stops at the
-// problem it belongs to and no carry crosses problems.  Small N therefore costs no extra
-// launches and rows need not be 16-byte aligned (only the base pointers).
+// cut into tiles; a tile that contains a problem start publishes its (trailing-segment)
+// inclusive value immediately, so every look-back stops inside its own problem and no
+// carry crosses problems.  Small N costs no extra launches and rows need not be 16-byte
+// aligned (only the base pointers).
 //
-// Descriptor protocol (per tile t, reset-free thanks to a 30-bit epoch tag):
-//   packed (32-bit carries): u64 = value<<32 | tag<<2 | status   (status 0 X, 1 A, 2 P)
-//   split  (f32 add, fp64 carries): u64 tag<<2|status + f64 aggregate[t] + f64 inclusive[t];
-//          the value is written first, the status with st.release; readers ld.acquire.
-// Tiles are numbered by an atomic ticket in CTA start order (forward progress: every tile
-// a CTA waits on belongs to a CTA that already started).  The last CTA to finish resets
-// the ticket and done counters and advances the epoch, so consecutive launches (also CUDA
-// graph replays) need no memset.
+// B200 structure (variants 0-2, persistent + warp-specialised):
+//   * one producer warp per CTA takes tile tickets (atomic, so tiles are handed out in
+//     start order: every tile waited on is owned by a running CTA) and streams the tiles
+//     into an S-stage shared-memory ring with 1-D TMA bulk copies (cp.async.bulk, SASS
+//     UBLKCP) completing on mbarriers -- the bytes in flight are bounded by smem, not by
+//     registers;
+//   * WARPS consumer warps scan each staged tile in two passes over smem (pass 1 prefixes,
+//     look-back by the last warp, pass 2 outputs with 128-bit streaming stores) and free
+//     the stage through an "empty" mbarrier;
+//   * the look-back window is 32*M tiles wide (each lane inspects M descriptors per
+//     round trip): a single huge problem (configs[2], N = 2^30) advances its inclusive
+//     front by up to 128 tiles per L2 round trip instead of 32.
+// Variant 3 is a non-persistent one-tile-per-CTA TMA kernel, kept for comparison.
+//
+// Descriptors (one per tile; reset-free thanks to a 30-bit epoch tag in every word):
+//   word = payload32 << 32 | tag << 2 | status      status 0 X (not ready), 1 A, 2 P
+//   32-bit carries: one word;  fp64 carries (f32 add): two words (hi, lo halves of the
+//   double) written by one 128-bit store and read by one 128-bit load; a reader accepts
+//   the pair only if both tags are current and both statuses agree.  The payload is
+//   self-contained, so relaxed (.STRONG.GPU, L1-bypassing) accesses suffice.
+// The last CTA to finish resets the ticket / done counters and advances the epoch, so
+// consecutive launches (also CUDA-graph replays) need no memset.
 #include "scan_common.cuh"
 #include "scan_internal.h"
 
@@ -31,31 +45,49 @@ namespace {
 
 constexpr uint32_t ST_A = 1u, ST_P = 2u;
 constexpr uint32_t TAG_MASK = 0x3FFFFFFFu;
+constexpr int LB_M = 4;                      // descriptors per lane per look-back round trip
+
+int num_sms();
+
+__device__ __forceinline__ void st_relaxed_u64(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_v2u64(uint64_t* p, uint64_t a, uint64_t b) {
+    asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" :: "l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void ld_relaxed_v2u64(const uint64_t* p, uint64_t& a, uint64_t& b) {
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
 
 template <class Op>
 struct Desc {
     using C = typename Op::Carry;
     static __device__ __forceinline__ void publish(const LookbackParams& p, int64_t t, uint32_t tag,
                                                    uint32_t st, C v) {
-        if constexpr (Op::kSplitDesc) {
-            st_relaxed_f64((st == ST_P ? p.incl : p.agg) + t, v);
-            st_release_u64(p.desc + t, (uint64_t)((tag << 2) | st));
+        const uint64_t meta = (uint64_t)((tag << 2) | st);
+        if constexpr (sizeof(C) == 8) {
+            const uint64_t b = (uint64_t)__double_as_longlong(v);
+            st_relaxed_v2u64(p.desc + 2 * t, (b & 0xFFFFFFFF00000000ull) | meta, (b << 32) | meta);
         } else {
-            uint64_t w = ((uint64_t)to_bits<C>(v) << 32) | (uint64_t)((tag << 2) | st);
-            st_release_u64(p.desc + t, w);
+            st_relaxed_u64(p.desc + t, ((uint64_t)to_bits<C>(v) << 32) | meta);
         }
     }
-    // returns status (0 when stale / not yet written) and the matching value
+    // returns status (0 when stale, torn or not yet written) and the matching value
     static __device__ __forceinline__ uint32_t read(const LookbackParams& p, int64_t t, uint32_t tag, C& v) {
-        if constexpr (Op::kSplitDesc) {
-            uint64_t w = ld_acquire_u64(p.desc + t);
-            uint32_t s = (uint32_t)w;
-            if ((s >> 2) != tag || (w >> 32) != 0ull) return 0u;
-            uint32_t st = s & 3u;
-            v = ld_relaxed_f64((st == ST_P ? p.incl : p.agg) + t);
-            return st;
+        if constexpr (sizeof(C) == 8) {
+            uint64_t hi, lo;
+            ld_relaxed_v2u64(p.desc + 2 * t, hi, lo);
+            const uint32_t mh = (uint32_t)hi, ml = (uint32_t)lo;
+            if ((mh >> 2) != tag || mh != ml) return 0u;
+            v = __longlong_as_double((long long)((hi & 0xFFFFFFFF00000000ull) | (lo >> 32)));
+            return mh & 3u;
         } else {
-            uint64_t w = ld_acquire_u64(p.desc + t);
+            const uint64_t w = ld_relaxed_u64(p.desc + t);
             if ((((uint32_t)w) >> 2) != tag) return 0u;
             v = from_bits<C>((uint32_t)(w >> 32));
             return (uint32_t)w & 3u;
@@ -63,65 +95,91 @@ struct Desc {
     }
 };
 
-// Warp-cooperative look-back for tile `t` (t > first tile of its problem).  Lane i inspects
-// predecessor t-1-i; the window slides back 32 tiles at a time until an inclusive (P)
-// descriptor is found.  Only the lanes up to the nearest P are waited for.
-template <class Op>
+// Warp-cooperative look-back for tile `t` (t is not the first tile of its problem).  Each
+// round trip inspects the 32*LB_M nearest unvisited predecessors (lane l, slot m looks at
+// distance l + 32 m); it waits only for the predecessors up to the nearest inclusive (P)
+// one, folds their values and stops there, or slides the window further back.
+template <class Op, int M = LB_M>
 __device__ __forceinline__ typename Op::Carry look_back(const LookbackParams& p, int64_t t, uint32_t tag) {
     using C = typename Op::Carry;
     const int lane = lane_id();
     C run = Op::cidentity();
-    int64_t pred = t - 1 - lane;
+    int64_t front = t - 1;                  // nearest predecessor not yet folded
     while (true) {
-        C v = Op::cidentity();
-        uint32_t st;
-        unsigned pm;
-        int fp;
+        C v[M];
+        uint32_t st[M];
+        int dP;
         int spins = 0;
         while (true) {
-            st = pred >= 0 ? Desc<Op>::read(p, pred, tag, v) : ST_P;   // (never needed: tile 0 starts a problem)
-            pm = __ballot_sync(FULL, st == ST_P);
-            unsigned xm = __ballot_sync(FULL, st == 0u);
-            fp = pm ? (__ffs(pm) - 1) : 32;
-            unsigned need = fp >= 32 ? FULL : ((1u << fp) - 1u);
-            if ((xm & need) == 0u) break;
-            if (++spins > 4) __nanosleep(64);
+#pragma unroll
+            for (int m = 0; m < M; ++m) {
+                const int64_t pred = front - lane - 32 * m;
+                v[m] = Op::cidentity();
+                st[m] = pred >= 0 ? Desc<Op>::read(p, pred, tag, v[m]) : ST_P;
+            }
+            dP = 1 << 30;                    // distance of the nearest P in the window
+#pragma unroll
+            for (int m = M - 1; m >= 0; --m) {
+                const unsigned pm = __ballot_sync(FULL, st[m] == ST_P);
+                if (pm) dP = 32 * m + __ffs(pm) - 1;
+            }
+            bool ok = true;
+#pragma unroll
+            for (int m = 0; m < M; ++m) {
+                const unsigned xm = __ballot_sync(FULL, st[m] == 0u && (lane + 32 * m) < dP);
+                ok = ok && (xm == 0u);
+            }
+            if (ok) break;
+            if (++spins > 2) __nanosleep(32);
         }
-        C mine = (lane <= fp && pred >= 0) ? v : Op::cidentity();
-        C w = warp_reduce_carry<Op>(mine);
-        run = Op::capply(w, run);          // the window is older than what we have so far
-        if (pm) break;
-        pred -= 32;
+        C mine = Op::cidentity();
+#pragma unroll
+        for (int m = 0; m < M; ++m)
+            if (lane + 32 * m <= dP && front - lane - 32 * m >= 0) mine = Op::capply(v[m], mine);
+        run = Op::capply(warp_reduce_carry<Op>(mine), run);   // the window is older than `run`
+        if (dP < (1 << 30)) break;
+        front -= 32 * M;
     }
     return run;
 }
 
-template <class Op, bool SEG, int WARPS, int V>
-__device__ __forceinline__ void tile_body(const LookbackParams& p, int64_t tile, uint32_t tag,
-                                          int64_t r, typename Op::Carry* s_carry,
-                                          typename Op::T* s_wval, uint32_t* s_wflag) {
+// debug timeline (scan_debug_trace): stamp e of tile t with %globaltimer (ns)
+__device__ __forceinline__ void trace_stamp(const LookbackParams& p, int64_t t, int e) {
+    if (p.trace != nullptr && t < p.trace_tiles) {
+        uint64_t g;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        p.trace[4 * t + e] = g;
+    }
+}
+
+__device__ __forceinline__ void consumer_bar(int nthreads) {
+    asm volatile("bar.sync 1, %0;" :: "r"(nthreads) : "memory");
+}
+
+// Tile body with the tile already in shared memory: pass 1, look-back by the last warp,
+// pass 2.  With NAMED_BAR only the WARPS consumer warps synchronise.
+template <class Op, bool SEG, int WARPS, int V, bool NAMED_BAR>
+__device__ __forceinline__ void tile_body_smem(const LookbackParams& p, int64_t tile, uint32_t tag, int64_t r,
+                                               const typename Op::T* s_tile, bool fast,
+                                               typename Op::Carry* s_carry, typename Op::T* s_wval,
+                                               uint32_t* s_wflag) {
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4;
     constexpr int WCH = V * 128;
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t base = tile * (int64_t)TILE;
-    const int64_t wbase = base + warp * WCH;
-    const T* in = (const T*)p.in;
-    T* out = (T*)p.out;
+    const T* srow = s_tile + warp * WCH;
 
-    WarpTile<Op, SEG, V> wt;
-    wt.load(in, wbase, p.total, p.vec);
-    if (SEG) {
+    WarpTileS<Op, SEG, V> wt;
+    {
         const bool small = p.N < TILE;
         int first = -1;
-        if (!small) first = r == 0 ? 0 : (int)(p.N - r);      // < TILE: SEG implies a head in the tile
-        wt.heads(warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+        if (SEG && !small) first = r == 0 ? 0 : (int)(p.N - r);   // < TILE: SEG implies a head here
+        wt.pass1(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
     }
-    wt.scan();
     if (lane == 0) { s_wval[warp] = wt.wtot; s_wflag[warp] = wt.wfl; }
-    __syncthreads();
-
+    if (NAMED_BAR) consumer_bar(WARPS * 32); else __syncthreads();
     T wp = Op::identity(); bool wpf = false;
 #pragma unroll
     for (int w = 0; w < WARPS; ++w) {
@@ -131,9 +189,7 @@ __device__ __forceinline__ void tile_body(const LookbackParams& p, int64_t tile,
             wpf = wpf || f;
         }
     }
-
     if (warp == WARPS - 1) {
-        // tile aggregate = (warps < last) . (last warp)
         T agg = SEG ? seg_fold<Op>(wp, wt.wfl, wt.wtot) : Op::apply(wp, wt.wtot);
         const bool starts = (r == 0);
         const bool has_head = SEG ? (wpf || wt.wfl) : starts;
@@ -146,89 +202,745 @@ __device__ __forceinline__ void tile_body(const LookbackParams& p, int64_t tile,
             *s_carry = carry;
         }
     }
-    __syncthreads();
+    if (NAMED_BAR) consumer_bar(WARPS * 32); else __syncthreads();
     const T cin = Op::from_carry(*s_carry);
-    wt.store(out, wbase, p.total, p.vec, wp, wpf, cin, p.exclusive);
+    wt.pass2(srow, (T*)p.out, base + warp * WCH, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
 }
 
-template <class Op, int WARPS, int V>
-__global__ void __launch_bounds__(WARPS * 32) lookback_kernel(LookbackParams p) {
+// Tile classification done once per tile by whoever owns the ticket.
+struct TileInfo { int64_t r; uint32_t seg; uint32_t fast; };
+__device__ __forceinline__ TileInfo classify(const LookbackParams& p, int64_t t, int tile_elems) {
+    TileInfo ti;
+    const int64_t base = t * (int64_t)tile_elems;
+    ti.r = base % p.N;
+    const int64_t count = p.total - base < tile_elems ? p.total - base : tile_elems;
+    const int64_t next_head = ti.r == 0 ? p.N : p.N - ti.r;    // first problem start after offset 0
+    ti.seg = next_head < count ? 1u : 0u;
+    ti.fast = (p.vec && count == tile_elems) ? 1u : 0u;
+    return ti;
+}
+
+// The last CTA to finish resets the counters and advances the epoch (wrap: clear all).
+__device__ __forceinline__ void epilogue(const LookbackParams& p) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(p.ctl + 1, 1u);
+    if (prev == gridDim.x - 1) {
+        __threadfence();
+        uint32_t e = *((volatile uint32_t*)(p.ctl + 2)) + 1u;
+        if (e + 1u >= TAG_MASK) {
+            for (int64_t i = 0; i < 2 * p.capacity; ++i) p.desc[i] = 0ull;
+            e = 0u;
+        }
+        ((volatile uint32_t*)p.ctl)[0] = 0u;
+        ((volatile uint32_t*)p.ctl)[1] = 0u;
+        ((volatile uint32_t*)p.ctl)[2] = e;
+        __threadfence();
+    }
+}
+
+__device__ __forceinline__ uint32_t read_tag(const LookbackParams& p) {
+    uint32_t e;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(e) : "l"(p.ctl + 2) : "memory");
+    return (e + 1u) & TAG_MASK;
+}
+
+
+// ---------------------------------------------------------------- persistent, warp-specialised
+template <class Op, int WARPS, int V, int S>
+__global__ void __launch_bounds__((WARPS + 1) * 32) lookback_persistent_kernel(LookbackParams p, int64_t num_tiles) {
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4;
-    __shared__ int64_t s_tile, s_r;
-    __shared__ uint32_t s_tag, s_seg;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    T* s_data = (T*)dsm;
+    __shared__ uint64_t s_full[S], s_empty[S];
+    __shared__ int64_t s_tid[S], s_r[S];
+    __shared__ uint32_t s_seg[S], s_fast[S];
+    __shared__ uint32_t s_tag;
     __shared__ C s_carry;
     __shared__ T s_wval[WARPS];
     __shared__ uint32_t s_wflag[WARPS];
-    __shared__ int s_last;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
 
     if (threadIdx.x == 0) {
-        int64_t t = (int64_t)atomicAdd(p.ctl + 0, 1u);
-        uint32_t e;
-        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(e) : "l"(p.ctl + 2) : "memory");
-        int64_t base = t * (int64_t)TILE;
-        int64_t r = base % p.N;
-        int64_t count = p.total - base < TILE ? p.total - base : TILE;
-        int64_t next_head = r == 0 ? p.N : p.N - r;          // first head after offset 0
-        s_tile = t; s_r = r; s_tag = (e + 1u) & TAG_MASK;
-        s_seg = next_head < count ? 1u : 0u;
+#pragma unroll
+        for (int s = 0; s < S; ++s) { mbar_init(&s_full[s], 1); mbar_init(&s_empty[s], WARPS); }
+        fence_mbar_init();
+        s_tag = read_tag(p);
     }
     __syncthreads();
-    const int64_t tile = s_tile, r = s_r;
     const uint32_t tag = s_tag;
-    if (s_seg) tile_body<Op, true, WARPS, V>(p, tile, tag, r, &s_carry, s_wval, s_wflag);
-    else       tile_body<Op, false, WARPS, V>(p, tile, tag, r, &s_carry, s_wval, s_wflag);
 
-    // ---- self-cleaning epilogue: the last CTA resets the counters and advances the epoch
-    if (threadIdx.x == 0) {
-        __threadfence();
-        uint32_t prev = atomicAdd(p.ctl + 1, 1u);
-        s_last = (prev == gridDim.x - 1) ? 1 : 0;
-        if (s_last) {
-            __threadfence();
-            uint32_t e = *((volatile uint32_t*)(p.ctl + 2)) + 1u;
-            bool wrap = e + 1u >= TAG_MASK;
-            if (wrap) {
-                // once every 2^30 launches: invalidate every descriptor ever written
-                for (int64_t i = 0; i < p.capacity; ++i) p.desc[i] = 0ull;
-                e = 0u;
+    if (warp == WARPS) {
+        // ---------------- producer warp: this CTA's tiles (round robin) into the TMA ring
+        const T* in = (const T*)p.in;
+        const uint64_t pol = l2_evict_first_policy();
+        int stage = 0;
+        uint32_t phase = 0;
+        for (int64_t t = blockIdx.x;; t += gridDim.x) {
+            mbar_wait(&s_empty[stage], phase ^ 1u);             // consumers freed this slot
+            if (t >= num_tiles) {
+                if (lane == 0) { s_tid[stage] = -1; mbar_arrive(&s_full[stage]); }
+                break;
             }
-            ((volatile uint32_t*)p.ctl)[0] = 0u;
-            ((volatile uint32_t*)p.ctl)[1] = 0u;
-            ((volatile uint32_t*)p.ctl)[2] = e;
-            __threadfence();
+            const TileInfo ti = classify(p, t, TILE);
+            T* dst = s_data + (size_t)stage * TILE;
+            const int64_t base = t * (int64_t)TILE;
+            if (lane == 0) { s_tid[stage] = t; s_r[stage] = ti.r; s_seg[stage] = ti.seg; s_fast[stage] = ti.fast; }
+            if (ti.fast) {
+                if (lane == 0) {
+                    mbar_expect_tx(&s_full[stage], TILE * 4);
+                    tma_load_1d(dst, in + base, TILE * 4, &s_full[stage], pol);
+                }
+            } else {
+                // ragged tail tile or unaligned base pointers: guarded copy, identity padding
+                for (int i = lane; i < TILE; i += 32)
+                    dst[i] = base + i < p.total ? from_bits<T>(ld_stream_u32(in + base + i)) : Op::identity();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&s_full[stage]);
+            }
+            if (++stage == S) { stage = 0; phase ^= 1u; }
         }
+    } else {
+        // ---------------- consumer warps
+        int stage = 0;
+        uint32_t phase = 0;
+        while (true) {
+            mbar_wait(&s_full[stage], phase);
+            const int64_t t = s_tid[stage];
+            if (t < 0) break;
+            const int64_t r = s_r[stage];
+            const bool fast = s_fast[stage] != 0u;
+            const T* st = s_data + (size_t)stage * TILE;
+            if (s_seg[stage]) tile_body_smem<Op, true, WARPS, V, true>(p, t, tag, r, st, fast, &s_carry, s_wval, s_wflag);
+            else              tile_body_smem<Op, false, WARPS, V, true>(p, t, tag, r, st, fast, &s_carry, s_wval, s_wflag);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&s_empty[stage]);
+            if (++stage == S) { stage = 0; phase ^= 1u; }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
+// ---------------------------------------------------------------- pipelined, dedicated look-back warp
+// Warp roles: WARPS consumer warps, one producer warp (TMA ring), one look-back warp.
+// Per ring slot: full (producer -> consumers), p1 (consumers' pass 1 done -> look-back
+// warp), cr (carry ready -> consumers), empty (consumers' pass 2 done -> producer).
+// Consumers run pass 1 of tile i+1 before pass 2 of tile i, so the look-back of tile i
+// (>= 1 L2 round trip) overlaps with useful work instead of idling 8 warps at a barrier.
+template <class Op, int WARPS>
+struct SlotHdr {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    int64_t tid;
+    int64_t r;
+    uint32_t seg, fast;
+    T wtot[WARPS];
+    uint32_t wfl[WARPS];
+    T wp[WARPS];
+    uint32_t wpf[WARPS];
+    C agg;
+    uint32_t has_head;
+    C carry;
+};
+
+template <class Op, int WARPS, int V, int S>
+struct PipeCtx {
+    using T = typename Op::T;
+    static constexpr int TILE = WARPS * 32 * V * 4;
+    static constexpr int WCH = V * 128;
+    T* data;
+    SlotHdr<Op, WARPS>* hdr;
+    uint64_t* full;
+    uint64_t* p1;
+    uint64_t* cr;
+    uint64_t* empty;
+};
+
+// consumer: pass 1 of the tile in sequence slot i; false at the end sentinel
+// The aggregate (A) -- or, for a tile holding a problem start, the inclusive value (P) --
+// is published right here by the last consumer warp, not by the look-back warp: a tile's
+// A must never wait for the look-back of the CTA's previous tile, or every round of the
+// round-robin schedule would serialise behind the previous round's resolution.
+template <class Op, int WARPS, int V, int S>
+__device__ __forceinline__ bool pipe_pass1(const LookbackParams& p, const PipeCtx<Op, WARPS, V, S>& c,
+                                           WarpTileP<Op, V>& st, int64_t i, uint32_t tag) {
+    using T = typename Op::T;
+    constexpr int TILE = PipeCtx<Op, WARPS, V, S>::TILE, WCH = PipeCtx<Op, WARPS, V, S>::WCH;
+    const int slot = (int)(i % S);
+    const uint32_t ph = (uint32_t)((i / S) & 1);
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    mbar_wait(&c.full[slot], ph);
+    SlotHdr<Op, WARPS>& h = c.hdr[slot];
+    if (h.tid < 0) {
+        if (warp == WARPS - 1 && lane == 0) mbar_arrive(&c.p1[slot]);
+        return false;
+    }
+    if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 0);
+    const T* srow = c.data + (size_t)slot * TILE + warp * WCH;
+    const int64_t r = h.r;
+    if (h.seg) {
+        const bool small = p.N < TILE;
+        const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+        st.template pass1<true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+    } else {
+        st.template pass1<false>(srow, warp * WCH, false, 0u, 1u, -1);
+    }
+    if (lane == 0) {
+        h.wtot[warp] = st.wtot;
+        h.wfl[warp] = st.wfl ? 1u : 0u;
+    }
+    consumer_bar(WARPS * 32);
+    if (warp == WARPS - 1) {
+        const bool seg = h.seg != 0u;
+        T run = Op::identity(); bool f = false;
+#pragma unroll
+        for (int w = 0; w < WARPS; ++w) {                // segmented exclusive prefix of warp totals
+            if (lane == w) { h.wp[w] = run; h.wpf[w] = f ? 1u : 0u; }
+            const T v = h.wtot[w];
+            const bool fw = seg && h.wfl[w] != 0u;
+            run = fw ? v : Op::apply(run, v);
+            f = f || fw;
+        }
+        const bool has_head = seg ? f : (r == 0);
+        if (lane == 0) {
+            h.agg = Op::to_carry(run);
+            h.has_head = has_head ? 1u : 0u;
+            trace_stamp(p, h.tid, 1);
+            Desc<Op>::publish(p, h.tid, tag, has_head ? ST_P : ST_A, h.agg);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&c.p1[slot]);
+    }
+    return true;
+}
+
+// consumer: pass 2 of the tile in sequence slot i (carry from the look-back warp)
+template <class Op, int WARPS, int V, int S>
+__device__ __forceinline__ void pipe_pass2(const LookbackParams& p, const PipeCtx<Op, WARPS, V, S>& c,
+                                           const WarpTileP<Op, V>& st, int64_t i) {
+    using T = typename Op::T;
+    constexpr int TILE = PipeCtx<Op, WARPS, V, S>::TILE, WCH = PipeCtx<Op, WARPS, V, S>::WCH;
+    const int slot = (int)(i % S);
+    const uint32_t ph = (uint32_t)((i / S) & 1);
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    mbar_wait(&c.cr[slot], ph);
+    const SlotHdr<Op, WARPS>& h = c.hdr[slot];
+    const T* srow = c.data + (size_t)slot * TILE + warp * WCH;
+    const int64_t gidx = h.tid * (int64_t)TILE + warp * WCH;
+    const bool fast = h.fast != 0u;
+    const T cin = Op::from_carry(h.carry);
+    const T wp = h.wp[warp];
+    const bool wpf = h.wpf[warp] != 0u;
+    if (h.seg) st.template pass2<true>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+    else       st.template pass2<false>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+    __syncwarp();
+    if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 3);
+    if (lane == 0) mbar_arrive(&c.empty[slot]);
+}
+
+template <class Op, int WARPS, int V, int S, int M>
+__global__ void __launch_bounds__((WARPS + 2) * 32) lookback_pipelined_kernel(LookbackParams p, int64_t num_tiles) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    using Ctx = PipeCtx<Op, WARPS, V, S>;
+    constexpr int TILE = Ctx::TILE;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    __shared__ SlotHdr<Op, WARPS> s_hdr[S];
+    __shared__ uint64_t s_full[S], s_p1[S], s_cr[S], s_empty[S];
+    __shared__ uint32_t s_tag;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    Ctx c{(T*)dsm, s_hdr, s_full, s_p1, s_cr, s_empty};
+
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&s_full[s], 1); mbar_init(&s_p1[s], 1);
+            mbar_init(&s_cr[s], 1);   mbar_init(&s_empty[s], WARPS);
+        }
+        fence_mbar_init();
+        s_tag = read_tag(p);
+    }
+    __syncthreads();
+    const uint32_t tag = s_tag;
+
+    if (warp < WARPS) {
+        // ---------------- consumers: pass1(i+1) then pass2(i), two register states
+        WarpTileP<Op, V> A, B;
+        int64_t i = 0;
+        if (pipe_pass1<Op, WARPS, V, S>(p, c, A, 0, tag)) {
+            while (true) {
+                ++i;
+                bool more = pipe_pass1<Op, WARPS, V, S>(p, c, B, i, tag);
+                pipe_pass2<Op, WARPS, V, S>(p, c, A, i - 1);
+                if (!more) break;
+                ++i;
+                more = pipe_pass1<Op, WARPS, V, S>(p, c, A, i, tag);
+                pipe_pass2<Op, WARPS, V, S>(p, c, B, i - 1);
+                if (!more) break;
+            }
+        }
+    } else if (warp == WARPS) {
+        // ---------------- producer: this CTA's tiles (round robin) into the TMA ring
+        const T* in = (const T*)p.in;
+        const uint64_t pol = l2_evict_first_policy();
+        int64_t i = 0;
+        for (int64_t t = blockIdx.x;; t += gridDim.x, ++i) {
+            const int slot = (int)(i % S);
+            const uint32_t ph = (uint32_t)((i / S) & 1);
+            mbar_wait(&s_empty[slot], ph ^ 1u);
+            SlotHdr<Op, WARPS>& h = s_hdr[slot];
+            if (t >= num_tiles) {
+                if (lane == 0) { h.tid = -1; mbar_arrive(&s_full[slot]); }
+                break;
+            }
+            const TileInfo ti = classify(p, t, TILE);
+            T* dst = c.data + (size_t)slot * TILE;
+            const int64_t base = t * (int64_t)TILE;
+            if (lane == 0) { h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast; }
+            if (ti.fast) {
+                if (lane == 0) {
+                    mbar_expect_tx(&s_full[slot], TILE * 4);
+                    tma_load_1d(dst, in + base, TILE * 4, &s_full[slot], pol);
+                }
+            } else {
+                for (int k = lane; k < TILE; k += 32)
+                    dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&s_full[slot]);
+            }
+        }
+    } else {
+        // ---------------- look-back warp: warp prefixes, publish, look back, carry
+        for (int64_t i = 0;; ++i) {
+            const int slot = (int)(i % S);
+            const uint32_t ph = (uint32_t)((i / S) & 1);
+            mbar_wait(&s_p1[slot], ph);
+            SlotHdr<Op, WARPS>& h = s_hdr[slot];
+            const int64_t t = h.tid;
+            if (t < 0) break;
+            const bool starts = (h.r == 0);
+            const bool has_head = h.has_head != 0u;
+            const C aggc = h.agg;
+            C carry = Op::cidentity();
+            if (!starts) carry = look_back<Op, M>(p, t, tag);
+            if (lane == 0) {
+                if (!has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, aggc));
+                h.carry = carry;
+                trace_stamp(p, t, 2);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&s_cr[slot]);
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
+// ---------------------------------------------------------------- two reads, L2-staged (variant 0)
+// Little's law: a tile that waits in shared memory for its carry holds a slot for the
+// whole look-back latency (several us under full HBM load), which caps a single huge
+// problem at ~5 TB/s.  Here the tile is read TWICE but from HBM only once:
+//   read 1 (TMA, HBM -> smem ring R, L2 evict_last)   reducer warps fold it, publish the
+//          aggregate (A) or, for a tile holding a problem start, the inclusive value (P);
+//          the R slot is released at once;
+//   look-back warp resolves the carry (no smem held while it waits);
+//   read 2 (TMA, L2 -> smem ring W, evict_first) issued once the carry is known: the
+//          tile is still L2-resident (a few MB in flight vs a 126 MB L2), so this read
+//          costs L2 bandwidth, not HBM; scanner warps scan it with the carry and store.
+// HBM traffic stays 2N; the look-back wait costs only a header slot.
+// Roles: NS scanner warps | NR reducer warps | P1 (read 1) | P2 (read 2) | LB.
+template <class Op, int V>
+__device__ __forceinline__ typename Op::T warp_reduce_rows(const typename Op::T* srow) {
+    using T = typename Op::T;
+    const int lane = lane_id();
+    T acc = Op::identity();
+#pragma unroll
+    for (int j = 0; j < V; ++j) {
+        Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+        acc = Op::apply(acc, Op::apply(Op::apply(x.v[0], x.v[1]), Op::apply(x.v[2], x.v[3])));
+    }
+#pragma unroll
+    for (int d = 16; d >= 1; d >>= 1) acc = Op::apply(acc, from_bits<T>(__shfl_xor_sync(FULL, to_bits<T>(acc), d)));
+    return acc;
+}
+
+// wait for an mbarrier phase, or give up once the end index (set by the reducers when they
+// meet the end sentinel) is < i; returns false in the latter case.  The warp that owns the
+// sentinel index itself (end == i) must wait: it forwards the sentinel to P2.
+__device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t phase, const int64_t* end, int64_t i) {
+    while (true) {
+        uint32_t ok;
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(ok) : "r"(smem_u32(bar)), "r"(phase) : "memory");
+        if (ok) return true;
+        if (*(const volatile int64_t*)end < i) return false;
     }
 }
 
-template <class Op, int WARPS, int V>
-cudaError_t launch_variant(const LookbackParams& p, cudaStream_t s) {
-    constexpr int TILE = WARPS * 32 * V * 4;
-    int64_t tiles = (p.total + TILE - 1) / TILE;
+template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
+__global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kernel(LookbackParams p, int64_t num_tiles) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int V = 8, WCH = V * 128, TILE = NS * WCH;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    T* bufR = (T*)dsm;                       // SR x TILE
+    T* bufW = bufR + (size_t)SR * TILE;      // SW x TILE
+    __shared__ SlotHdr<Op, NS> s_hdr[SH];
+    __shared__ uint64_t fullR[SR], emptyR[SR], fullW[SW], emptyW[SW], aggd[SH], crd[SH], emptyH[SH];
+    __shared__ uint32_t s_tag;
+    __shared__ int64_t s_end;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+
+    if (threadIdx.x == 0) {
+        s_end = INT64_MAX;
+        for (int s = 0; s < SR; ++s) { mbar_init(&fullR[s], 1); mbar_init(&emptyR[s], NR); }
+        for (int s = 0; s < SW; ++s) { mbar_init(&fullW[s], 1); mbar_init(&emptyW[s], NS); }
+        for (int s = 0; s < SH; ++s) { mbar_init(&aggd[s], 1); mbar_init(&crd[s], 1); mbar_init(&emptyH[s], NS); }
+        fence_mbar_init();
+        s_tag = read_tag(p);
+    }
+    __syncthreads();
+    const uint32_t tag = s_tag;
+    const T* in = (const T*)p.in;
+
+    if (warp < NS) {
+        // ---------------- scanners: read 2 landed -> full scan with the carry -> store
+        for (int64_t i = 0;; ++i) {
+            const int sW = (int)(i % SW), sH = (int)(i % SH);
+            mbar_wait(&fullW[sW], (uint32_t)((i / SW) & 1));
+            const SlotHdr<Op, NS>& h = s_hdr[sH];
+            const int64_t t = h.tid;
+            if (t < 0) break;
+            const T* srow = bufW + (size_t)sW * TILE + warp * WCH;
+            const T cin = Op::from_carry(h.carry);
+            const T wp = h.wp[warp];
+            const bool wpf = h.wpf[warp] != 0u, fast = h.fast != 0u;
+            const int64_t gidx = t * (int64_t)TILE + warp * WCH;
+            WarpTileP<Op, V> st;
+            if (h.seg) {
+                const int64_t r = h.r;
+                const bool small = p.N < TILE;
+                const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+                st.template pass1<true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+                st.template pass2<true>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+            } else {
+                st.template pass1<false>(srow, warp * WCH, false, 0u, 1u, -1);
+                st.template pass2<false>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+            }
+            __syncwarp();
+            if (lane == 0) {
+                if (warp == 0) trace_stamp(p, t, 3);
+                mbar_arrive(&emptyW[sW]);
+                mbar_arrive(&emptyH[sH]);
+            }
+        }
+    } else if (warp < NS + NR) {
+        // ---------------- reducers: read 1 landed -> per-1024 totals -> A (or P)
+        const int rr = warp - NS;
+        for (int64_t i = 0;; ++i) {
+            const int sR = (int)(i % SR), sH = (int)(i % SH);
+            mbar_wait(&fullR[sR], (uint32_t)((i / SR) & 1));
+            SlotHdr<Op, NS>& h = s_hdr[sH];
+            const int64_t t = h.tid;
+            if (t < 0) {
+                if (rr == NR - 1 && lane == 0) {
+                    *(volatile int64_t*)&s_end = i;      // look-back warps waiting beyond i leave
+                    mbar_arrive(&aggd[sH]);
+                }
+                break;
+            }
+            if (rr == NR - 1 && lane == 0) trace_stamp(p, t, 0);
+            const bool seg = h.seg != 0u;
+            const int64_t r = h.r;
+            for (int k = rr; k < NS; k += NR) {
+                const T* srow = bufR + (size_t)sR * TILE + k * WCH;
+                T tot; bool fl = false;
+                if (seg) {
+                    const bool small = p.N < TILE;
+                    const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+                    WarpTileP<Op, V> st;
+                    st.template pass1<true>(srow, k * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+                    tot = st.wtot; fl = st.wfl;
+                } else {
+                    tot = warp_reduce_rows<Op, V>(srow);
+                }
+                if (lane == 0) { h.wtot[k] = tot; h.wfl[k] = fl ? 1u : 0u; }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&emptyR[sR]);
+            asm volatile("bar.sync 2, %0;" :: "r"(NR * 32) : "memory");
+            if (rr == NR - 1) {
+                T run = Op::identity(); bool f = false;
+#pragma unroll
+                for (int w = 0; w < NS; ++w) {
+                    if (lane == w) { h.wp[w] = run; h.wpf[w] = f ? 1u : 0u; }
+                    const T v = h.wtot[w];
+                    const bool fw = seg && h.wfl[w] != 0u;
+                    run = fw ? v : Op::apply(run, v);
+                    f = f || fw;
+                }
+                const bool has_head = seg ? f : (r == 0);
+                if (lane == 0) {
+                    h.agg = Op::to_carry(run);
+                    h.has_head = has_head ? 1u : 0u;
+                    Desc<Op>::publish(p, t, tag, has_head ? ST_P : ST_A, h.agg);
+                    trace_stamp(p, t, 1);
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&aggd[sH]);
+            }
+        }
+    } else if (warp == NS + NR) {
+        // ---------------- P1: read 1 of this CTA's tiles (round robin) into ring R
+        const uint64_t pol = l2_evict_last_policy();
+        int64_t i = 0;
+        for (int64_t t = blockIdx.x;; t += gridDim.x, ++i) {
+            const int sR = (int)(i % SR), sH = (int)(i % SH);
+            mbar_wait(&emptyR[sR], (uint32_t)((i / SR) & 1) ^ 1u);
+            mbar_wait(&emptyH[sH], (uint32_t)((i / SH) & 1) ^ 1u);
+            SlotHdr<Op, NS>& h = s_hdr[sH];
+            if (t >= num_tiles) {
+                if (lane == 0) { h.tid = -1; mbar_arrive(&fullR[sR]); }
+                break;
+            }
+            const TileInfo ti = classify(p, t, TILE);
+            T* dst = bufR + (size_t)sR * TILE;
+            const int64_t base = t * (int64_t)TILE;
+            if (lane == 0) { h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast; }
+            if (ti.fast) {
+                if (lane == 0) {
+                    mbar_expect_tx(&fullR[sR], TILE * 4);
+                    tma_load_1d(dst, in + base, TILE * 4, &fullR[sR], pol);
+                }
+            } else {
+                for (int k = lane; k < TILE; k += 32)
+                    dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&fullR[sR]);
+            }
+        }
+    } else if (warp == NS + NR + 1) {
+        // ---------------- P2: read 2 (from L2) once the carry is known, into ring W
+        const uint64_t pol = l2_evict_first_policy();
+        for (int64_t i = 0;; ++i) {
+            const int sW = (int)(i % SW), sH = (int)(i % SH);
+            mbar_wait(&crd[sH], (uint32_t)((i / SH) & 1));
+            mbar_wait(&emptyW[sW], (uint32_t)((i / SW) & 1) ^ 1u);
+            const SlotHdr<Op, NS>& h = s_hdr[sH];
+            const int64_t t = h.tid;
+            if (t < 0) {
+                if (lane == 0) mbar_arrive(&fullW[sW]);
+                break;
+            }
+            T* dst = bufW + (size_t)sW * TILE;
+            const int64_t base = t * (int64_t)TILE;
+            if (h.fast) {
+                if (lane == 0) {
+                    mbar_expect_tx(&fullW[sW], TILE * 4);
+                    tma_load_1d(dst, in + base, TILE * 4, &fullW[sW], pol);
+                }
+            } else {
+                for (int k = lane; k < TILE; k += 32)
+                    dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&fullW[sW]);
+            }
+        }
+    } else {
+        // ---------------- NLB look-back warps, tile sequence i handled by warp i mod NLB
+        const int lb = warp - (NS + NR + 2);
+        for (int64_t i = lb;; i += NLB) {
+            const int sH = (int)(i % SH);
+            if (!mbar_wait_or_end(&aggd[sH], (uint32_t)((i / SH) & 1), &s_end, i)) break;
+            SlotHdr<Op, NS>& h = s_hdr[sH];
+            const int64_t t = h.tid;
+            if (t < 0) {
+                if (lane == 0) mbar_arrive(&crd[sH]);
+                break;
+            }
+            C carry = Op::cidentity();
+            if (h.r != 0) carry = look_back<Op, M>(p, t, tag);
+            if (lane == 0) {
+                if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
+                h.carry = carry;
+                trace_stamp(p, t, 2);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&crd[sH]);
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
+template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
+cudaError_t launch_l2(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = NS * 1024;
+    constexpr int SMEM = (SR + SW) * TILE * 4;
+    constexpr int THREADS = (NS + NR + 2 + NLB) * 32;
+    auto kern = lookback_l2_kernel<Op, NS, NR, SR, SW, SH, M, NLB>;
+    static int occ = 0;
+    if (occ == 0) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        if (e != cudaSuccess) return e;
+        int o = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
+        if (e != cudaSuccess) return e;
+        if (o < 1) return cudaErrorInvalidConfiguration;
+        occ = o;
+    }
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
     if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    lookback_kernel<Op, WARPS, V><<<(unsigned)tiles, WARPS * 32, 0, s>>>(p);
+    int64_t grid = (int64_t)occ * num_sms();
+    if (grid > tiles) grid = tiles;
+    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- one tile per CTA (comparison)
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4;
+    constexpr int WCH = V * 128;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    T* s_tile = (T*)dsm;
+    __shared__ uint64_t s_bar[WARPS];
+    __shared__ int64_t s_tile_id, s_r;
+    __shared__ uint32_t s_tag, s_seg, s_fast;
+    __shared__ C s_carry;
+    __shared__ T s_wval[WARPS];
+    __shared__ uint32_t s_wflag[WARPS];
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+
+    // tiles follow blockIdx (blocks are dispatched in index order, so every tile a CTA
+    // waits on belongs to a CTA that is already running); the bulk copy of each warp's
+    // share is issued first, the bookkeeping overlaps with it
+    const int64_t tile = blockIdx.x;
+    const int64_t base = tile * (int64_t)TILE;
+    const bool fast = p.vec && base + TILE <= p.total;
+    const T* in = (const T*)p.in;
+    if (fast && lane == 0) {
+        mbar_init(&s_bar[warp], 1);
+        fence_mbar_init();
+        mbar_expect_tx(&s_bar[warp], WCH * 4);
+        tma_load_1d(s_tile + warp * WCH, in + base + warp * WCH, WCH * 4, &s_bar[warp], l2_evict_first_policy());
+    }
+    if (threadIdx.x == 0) {
+        const TileInfo ti = classify(p, tile, TILE);
+        s_tile_id = tile; s_r = ti.r; s_seg = ti.seg; s_fast = ti.fast;
+        s_tag = read_tag(p);
+    }
+    __syncthreads();
+    const int64_t r = s_r;
+    const uint32_t tag = s_tag;
+    if (fast) {
+        mbar_wait(&s_bar[warp], 0);
+    } else {
+        for (int i = threadIdx.x; i < TILE; i += WARPS * 32)
+            s_tile[i] = base + i < p.total ? from_bits<T>(ld_stream_u32(in + base + i)) : Op::identity();
+        __syncthreads();
+    }
+    if (s_seg) tile_body_smem<Op, true, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
+    else       tile_body_smem<Op, false, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
+// ---------------------------------------------------------------- launchers
+int g_num_sms = 0;
+
+int num_sms() {
+    if (g_num_sms == 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+        if (g_num_sms <= 0) g_num_sms = 148;
+    }
+    return g_num_sms;
+}
+
+template <class Op, int WARPS, int V, int S>
+cudaError_t launch_persistent(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = WARPS * 32 * V * 4;
+    constexpr int SMEM = S * TILE * 4;
+    constexpr int THREADS = (WARPS + 1) * 32;
+    auto kern = lookback_persistent_kernel<Op, WARPS, V, S>;
+    static int occ = 0;                       // per instantiation; computed once
+    if (occ == 0) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        if (e != cudaSuccess) return e;
+        int o = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
+        if (e != cudaSuccess) return e;
+        if (o < 1) return cudaErrorInvalidConfiguration;
+        occ = o;
+    }
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    int64_t grid = (int64_t)occ * num_sms();
+    if (grid > tiles) grid = tiles;
+    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
+    return cudaGetLastError();
+}
+
+template <class Op, int WARPS, int V>
+cudaError_t launch_tma(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = WARPS * 32 * V * 4;
+    constexpr int SMEM = TILE * 4;
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    if (SMEM > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(lookback_tma_kernel<Op, WARPS, V>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        if (e != cudaSuccess) return e;
+    }
+    lookback_tma_kernel<Op, WARPS, V><<<(unsigned)tiles, WARPS * 32, SMEM, s>>>(p);
+    return cudaGetLastError();
+}
+
+template <class Op, int WARPS, int V, int S, int M>
+cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = WARPS * 32 * V * 4;
+    constexpr int SMEM = S * TILE * 4;
+    constexpr int THREADS = (WARPS + 2) * 32;
+    auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M>;
+    static int occ = 0;
+    if (occ == 0) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        if (e != cudaSuccess) return e;
+        int o = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
+        if (e != cudaSuccess) return e;
+        if (o < 1) return cudaErrorInvalidConfiguration;
+        occ = o;
+    }
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    int64_t grid = (int64_t)occ * num_sms();
+    if (grid > tiles) grid = tiles;
+    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
     return cudaGetLastError();
 }
 
 template <class Op>
 cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     switch (variant) {
-    case 0: return launch_variant<Op, 8, 4>(p, s);     // 4096-element tiles
-    case 1: return launch_variant<Op, 8, 8>(p, s);     // 8192-element tiles
-    default: return launch_variant<Op, 16, 4>(p, s);   // 8192-element tiles, 16 warps
+    case 0: return launch_pipelined<Op, 16, 8, 3, 5>(p, s);     // 16384-element tiles (64 KiB), window 160
+    case 1: return launch_pipelined<Op, 8, 8, 3, 4>(p, s);      // 8192-element tiles, 3 x 32 KiB ring
+    case 2: return launch_l2<Op, 8, 4, 3, 3, 32, 4, 4>(p, s);   // two reads (L2-staged), 8192-element tiles
+    default: return launch_tma<Op, 8, 8>(p, s);                 // one 8192-element tile per CTA
     }
 }
 
 }  // namespace
 
-int64_t lookback_tile_elems(int variant) {
-    switch (variant) {
-    case 0: return 8 * 32 * 4 * 4;
-    case 1: return 8 * 32 * 8 * 4;
-    default: return 16 * 32 * 4 * 4;
-    }
-}
+int64_t lookback_tile_elems(int variant) { return variant == 0 ? 16384 : 8192; }
+int lookback_num_variants() { return 4; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

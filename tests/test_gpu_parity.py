@@ -39,7 +39,7 @@ def test_shapes_all_algos(algo, op, dt, kind):
             assert_parity(got, x, op, kind, label="%s %s %s %s N=%d G=%d" % (algo, op, dt, kind, N, G))
 
 
-@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3])
 def test_lookback_variants(variant):
     for op, dt in COMBOS:
         for N, G in [(1, 3000), (3, 5000), (100, 333), (8193, 5), (65536 + 17, 3), (1 << 20, 1)]:
@@ -232,16 +232,20 @@ def test_sharded_loopback_elements_mode():
             Ntot = sum(lens)
             x = inputs.generate(DIST[dt], G * Ntot, seed=len(lens) * 7 + G).reshape(G, Ntot)
             for kind in ("inclusive", "exclusive"):
-                parts, totals = [], []
+                parts, totals, wss = [], [], []
                 starts = np.cumsum([0] + lens)
                 for r, L in enumerate(lens):
                     xl = to_device(np.ascontiguousarray(x[:, starts[r]: starts[r] + L]))
-                    totals.append(sb.shard_totals(xl, op))
+                    # each virtual rank keeps its own workspace (its chunk prefixes) between
+                    # the two steps, as each real rank does on its own device
+                    nb = int(sb._lib.lib.scan_shard_workspace_bytes(L, G))
+                    wss.append(torch.zeros((nb + 7) // 8, dtype=torch.int64, device="cuda"))
+                    totals.append(sb.shard_totals(xl, op, workspace=wss[-1]))
                     parts.append(xl)
                 all_t = torch.stack(totals)                     # [W][G]
                 outs = []
                 for r, xl in enumerate(parts):
-                    outs.append(sb.shard_scan(xl, all_t, r, len(lens), op, kind))
+                    outs.append(sb.shard_scan(xl, all_t, r, len(lens), op, kind, workspace=wss[r]))
                 torch.cuda.synchronize()
                 got = np.concatenate([to_host(o, NP[dt]).reshape(G, -1) for o in outs], axis=1)
                 assert_parity(got, x, op, kind, label="sharded %s %s %s lens=%s" % (op, dt, kind, lens))
