@@ -142,6 +142,20 @@ def timed_steps(sb, xs, outs, K, per_launch=False):
     return total_ms, launch_ms
 
 
+def kernel_times(sb, xs, outs, reps):
+    res = []
+    for i, (dt, op, kind) in enumerate(VARIANTS):
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        s0.record()
+        for _ in range(reps):
+            sb.scan(xs[dt], op, kind, out=outs[i])
+        s1.record()
+        torch.cuda.synchronize()
+        res.append(s0.elapsed_time(s1) / reps)
+    return res
+
+
 def e2e(sb, K=3):
     """The same step through the public host-buffer API: pinned host in -> scan -> host out."""
     import inputs
@@ -308,6 +322,7 @@ def main():
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the CPU oracle baseline (profiling runs)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -361,8 +376,9 @@ def main():
         t = torch.tensor([total_ms], device=dev)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         total_ms = float(t.item())
-    # per-launch durations (separate pass, same launches, events around each launch)
-    _, launch_ms = timed_steps(sb, xs, outs, max(10, args.steps // 10), per_launch=True)
+    # average launch duration of each scan kernel: `reps` back-to-back launches of the same
+    # call between two events on the launching stream (no events between launches)
+    launch_ms = kernel_times(sb, xs, outs, max(20, args.steps // 4))
 
     ms_step = total_ms / args.steps
     elems_step = len(VARIANTS) * G_C2 * N_C2 * world
@@ -370,6 +386,7 @@ def main():
     bytes_launch = 2 * 4 * G_C2 * N_C2
     dom = max(range(len(VARIANTS)), key=lambda i: launch_ms[i])
     achieved = bytes_launch / (launch_ms[dom] * 1e-3) / 1e9
+    algo, param = sb.plan(xs[VARIANTS[dom][0]], outs[dom])
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tpath):
@@ -386,8 +403,10 @@ def main():
                              "frac": elems_step / world * 8 / (ms_step * 1e-3) / 1e9 / hbm, "peak_src": hbm_src},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "traffic": traffic,
-                     "kernel": "lookback_kernel (%s %s %s), %d B algorithmic per launch" % (
-                         VARIANTS[dom] + (bytes_launch,)),
+                     "kernel": "%s [algo=%s param=%d] on %s %s %s" % (
+                         sb.KERNEL_NAMES[algo], algo, param, *VARIANTS[dom]),
+                     "bytes_per_launch": bytes_launch, "ms_per_launch": launch_ms[dom],
+                     "bytes_basis": "2 x 4 B x G x N (read input once, write output once)",
                      "peak_src": hbm_src + " copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"},
         "per_launch_ms": {"%s_%s_%s" % v: m for v, m in zip(VARIANTS, launch_ms)},
         "gpu_launches": len(VARIANTS) * args.steps,
@@ -395,7 +414,7 @@ def main():
     }
     if rank == 0 and not args.no_e2e:
         res["e2e"] = e2e(sb)
-    if rank == 0 and world == 1:
+    if rank == 0 and world == 1 and not args.no_cpu:
         res["cpu_baseline"] = cpu_oracle_rate()
     if rank == 0 and world == 1 and not args.no_extras:
         del xs, outs

@@ -142,5 +142,21 @@ def shard_scan(x_local: torch.Tensor, all_totals: torch.Tensor, rank: int, ngpu:
     return out
 
 
+ALGO_NAMES = {v: k for k, v in ALGOS.items()}
+KERNEL_NAMES = {"lookback": "lookback_*_kernel (decoupled look-back)",
+                "cascade_cta": "chunk_scan_kernel (one CTA per problem, cascade)",
+                "cascade_warp": "warp_cascade_kernel (one warp per problem, cascade)",
+                "three_stage": "chunk_reduce + aux_scan + chunk_scan kernels"}
+
+
+def plan(x: torch.Tensor, out: torch.Tensor | None = None) -> tuple[str, int]:
+    """The (algo, param) that algo='auto' picks for this tensor (scan_plan)."""
+    N, G = _shape(x)
+    a, pr = ctypes.c_int(0), ctypes.c_int64(0)
+    check("scan_plan", _lib.lib.scan_plan(N, G, x.data_ptr(), (out if out is not None else x).data_ptr(),
+                                          ctypes.byref(a), ctypes.byref(pr)))
+    return ALGO_NAMES[a.value], pr.value
+
+
 def abi_version() -> int:
     return int(_lib.lib.scan_abi_version())

@@ -22,7 +22,9 @@ STATUS = {0: "SCAN_OK", 1: "SCAN_ERR_INVALID_ARG", 2: "SCAN_ERR_UNSUPPORTED", 3:
 # every symbol include/scan_b200.h declares (checked by tests/test_abi.py)
 EXPORTS = ("scan_status_string", "scan_abi_version", "scan_batch", "scan_workspace_bytes",
            "scan_batch_ex", "scan_batch_host", "scan_shard_totals", "scan_shard_scan",
-           "scan_shard_workspace_bytes", "scan_debug_trace")
+           "scan_shard_workspace_bytes", "scan_debug_trace", "scan_plan", "scan_comm_create_nccl",
+           "scan_comm_get_unique_id", "scan_comm_init_rank", "scan_comm_destroy", "scan_batch_multi")
+SHARD = {"problems": 0, "elements": 1}
 
 
 class ScanError(RuntimeError):
@@ -48,6 +50,12 @@ def _load() -> ctypes.CDLL:
         "scan_shard_scan": ([P, P, I64, I64, I, I, I, P, I, I, P, SZ, P], I),
         "scan_shard_workspace_bytes": ([I64, I64], SZ),
         "scan_debug_trace": ([P, I64], I),
+        "scan_plan": ([I64, I64, P, P, P, P], I),
+        "scan_comm_create_nccl": ([P, I, I, P], I),
+        "scan_comm_get_unique_id": ([P], I),
+        "scan_comm_init_rank": ([P, I, I, P], I),
+        "scan_comm_destroy": ([P], I),
+        "scan_batch_multi": ([P, P, I64, I64, I, I, I, P, I, P, I], I),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)

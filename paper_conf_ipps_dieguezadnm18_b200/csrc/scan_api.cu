@@ -368,6 +368,15 @@ scan_status scan_debug_trace(void* device_buf, int64_t tiles) {
     return SCAN_OK;
 }
 
+scan_status scan_plan(int64_t N, int64_t G, const void* in, const void* out, int* algo, int64_t* param) {
+    if (!algo || !param || N < 0 || G < 0) return SCAN_ERR_INVALID_ARG;
+    const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+    const scan_algo a = choose_algo(N, G, aligned);
+    *algo = (int)a;
+    *param = a == SCAN_ALGO_LOOKBACK ? choose_lookback_variant(N, G) : -1;
+    return SCAN_OK;
+}
+
 size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, scan_algo algo, int64_t param) {
     if (N <= 0 || G <= 0) return kCtlBytes;
     if (algo == SCAN_ALGO_AUTO) {

@@ -1,0 +1,109 @@
+"""Single-box multi-GPU scan: one process per GPU, torch.distributed for the plumbing.
+
+Two ways to use several GPUs (PAPER.md:191-193 [§4]):
+
+* ``mode="problems"`` -- Case 1: the G problems are split over the ranks
+  (:func:`partition`), every rank scans its own problems with the single-GPU kernels.
+  There is no communication at all ("Solving the Case 1 is trivial").
+* ``mode="elements"`` -- Case 2, Multi-GPU Problem Scattering (Figs.
+  6-7): every problem is split into rank-ordered contiguous portions.  Each rank runs
+  Stage 1+2 on its portion (``shard_totals``: chunk aggregates + one total per problem),
+  the totals of all ranks are exchanged with ONE all-gather of G 8-byte slots per rank
+  (NCCL over NVLink/NVSwitch -- the paper's P2P writes to a master GPU and its
+  MPI_Gather / MPI_Scatter, become a single collective, and every rank
+  folds the totals of the ranks before it itself), then Stage 3 (``shard_scan``) scans
+  the portion with that carry.  The output stays sharded like the input.
+
+``backend="torch"`` does the exchange with ``torch.distributed.all_gather_into_tensor``
+on the caller's process group; ``backend="native"`` calls the C-ABI
+``scan_batch_multi`` with the group's own NCCL communicator (one library call per rank).
+All device work runs in libscanb200.so; only the sharding plan and the collective call
+are Python.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+import torch.distributed as dist
+
+from . import _lib, shard_scan, shard_totals
+from ._lib import KINDS, OPS, check
+
+__all__ = ["partition", "exchange_totals", "scan_multi", "NativeComm"]
+
+
+def partition(n: int, world: int, rank: int) -> tuple[int, int]:
+    """Contiguous balanced split of n units: rank r owns [floor(r n / W), floor((r+1) n / W)).
+
+    Used for problems (Case 1) and for the elements of one problem (Case 2).  Any n >= 0 and
+    world >= 1 is legal; portions may be empty (the paper's Eqs. 2-3, PAPER.md:229-233,
+    become "any portion length is legal").
+    """
+    if world < 1 or not 0 <= rank < world or n < 0:
+        raise ValueError("bad partition arguments")
+    return (rank * n) // world, ((rank + 1) * n) // world
+
+
+def exchange_totals(totals: torch.Tensor, group=None) -> torch.Tensor:
+    """All-gather this rank's G total slots (int64) into a rank-major [W, G] tensor."""
+    world = dist.get_world_size(group)
+    src = totals.contiguous().view(-1)
+    out = torch.empty(world * src.numel(), dtype=totals.dtype, device=totals.device)
+    dist.all_gather_into_tensor(out, src, group=group)
+    return out.view((world,) + tuple(totals.shape))
+
+
+class NativeComm:
+    """scan_comm_t over the NCCL communicator of a torch ProcessGroupNCCL (borrowed)."""
+
+    def __init__(self, group=None):
+        pg = group if group is not None else dist.group.WORLD
+        backend = pg._get_backend(torch.device("cuda", torch.cuda.current_device()))
+        ptr = backend._comm_ptr()
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        h = ctypes.c_void_p(0)
+        check("scan_comm_create_nccl", _lib.lib.scan_comm_create_nccl(ctypes.c_void_p(ptr), self.rank,
+                                                                        self.world, ctypes.byref(h)))
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            check("scan_comm_destroy", _lib.lib.scan_comm_destroy(self.handle))
+            self.handle = None
+
+
+def scan_multi(x_local: torch.Tensor, op: str = "add", kind: str = "inclusive", mode: str = "elements",
+               group=None, out: torch.Tensor | None = None, backend: str = "torch",
+               comm: NativeComm | None = None) -> torch.Tensor:
+    """Scan this rank's share.  ``x_local`` is (G, N_local) or (N_local,).
+
+    mode="problems": x_local holds whole problems (this rank's partition of the batch).
+    mode="elements": x_local holds this rank's portion of each of the G problems.
+    Collective in elements mode: every rank of ``group`` must call it with the same G,
+    op, kind, mode and backend.
+    """
+    from . import scan as scan_local
+    if out is None:
+        out = torch.empty_like(x_local)
+    if mode == "problems":
+        return scan_local(x_local, op, kind, out=out)
+    if mode != "elements":
+        raise ValueError(mode)
+    if backend == "native":
+        c = comm if comm is not None else NativeComm(group)
+        N, G = (x_local.shape[0], 1) if x_local.dim() == 1 else (x_local.shape[1], x_local.shape[0])
+        from . import _dtype, _stream
+        rc = _lib.lib.scan_batch_multi(x_local.data_ptr(), out.data_ptr(), N, G, OPS[op], _dtype(x_local),
+                                       KINDS[kind], _stream(x_local, None), c.world, c.handle,
+                                       _lib.SHARD["elements"])
+        check("scan_batch_multi", rc)
+        if comm is None:
+            torch.cuda.current_stream().synchronize()
+            c.close()
+        return out
+    totals = shard_totals(x_local, op)                        # Stage 1 + 2 (local)
+    all_totals = exchange_totals(totals, group)               # the one exchange step
+    return shard_scan(x_local, all_totals, dist.get_rank(group), dist.get_world_size(group),
+                      op, kind, out=out)                      # Stage 3 (local)
