@@ -205,6 +205,32 @@ def cpu_oracle_rate(budget_s: float = 12.0):
             "ms_per_step": t_scan / steps * 1e3}
 
 
+def cpu_oracle_steps(steps: int, warmup: int, g_sample: int = 256):
+    """Reference arm: the oracle as it stands, `warmup` untimed + `steps` timed steps; each
+    step scans a bounded sample of the c2 batch (g_sample of its 4096 problems, all four
+    variants), so 200 steps stay within a few minutes on the host."""
+    import inputs
+    import oracle
+    xs = {dt: inputs.generate(DIST[dt], g_sample * N_C2, SEED + 2).reshape(g_sample, N_C2)
+          for dt in ("i32", "f32")}
+
+    def one():
+        for dt, op, kind in VARIANTS:
+            oracle.scan(xs[dt], op, kind)
+    for _ in range(warmup):
+        one()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        one()
+    t = time.perf_counter() - t0
+    elems = steps * len(VARIANTS) * g_sample * N_C2
+    return {"value": elems / t / 1e9, "unit": "Gelem/s", "cores": 1, "kind": "oracle",
+            "sample": "%d problems of the c2 batch (of 4096) x 4 variants per step, %d timed steps, "
+                      "single-threaded C oracle" % (g_sample, steps),
+            "host_cpu": _cpu_name(), "host_cores_available": len(os.sched_getaffinity(0)),
+            "ms_per_step": t / steps * 1e3}
+
+
 def _cpu_name():
     try:
         for line in open("/proc/cpuinfo"):
@@ -258,6 +284,49 @@ def extras(sb, dev):
     del x, y
     torch.cuda.empty_cache()
     return out
+
+
+def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
+    """configs[4]-style sharded single problem (Multi-GPU Problem Scattering):
+    each rank owns a contiguous 2^28-element int32 portion of ONE problem; Stage 1+2 ->
+    NCCL all-gather of the rank totals -> Stage 3.  Weak-scaled (N = W x 2^28).  At W = 1 the
+    same two-pass pipeline runs without the collective (its 1-GPU reference rate)."""
+    import inputs
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    x = torch.empty(n_local, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "i32", SEED + 5, offset=rank * n_local)
+    y = torch.empty_like(x)
+    comm = multi.NativeComm() if world > 1 else None
+
+    def run():
+        if world > 1:
+            multi.scan_multi(x, "add", "inclusive", mode="elements", out=y, backend="native", comm=comm)
+        else:
+            t = sb.shard_totals(x, "add")
+            sb.shard_scan(x, t.view(1, -1), 0, 1, "add", "inclusive", out=y)
+    for _ in range(3):
+        run()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    for _ in range(reps):
+        run()
+    s1.record()
+    torch.cuda.synchronize()
+    ms = s0.elapsed_time(s1) / reps
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+        comm.close()
+    hbm, _, _ = _peaks()
+    per_gpu_gbs = 12.0 * n_local / (ms * 1e-3) / 1e9          # reduce pass (4 B) + scan pass (8 B)
+    return {"N_total": world * n_local, "N_per_gpu": n_local, "ms": ms,
+            "Gelem/s": world * n_local / ms / 1e6, "per_gpu_GB/s_at_12B_per_elem": per_gpu_gbs,
+            "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
+            "exchange": "NCCL allgather (scan_batch_multi, native comm)" if world > 1 else "none (W=1)"}
 
 
 def sweep(sb, dev):
@@ -338,7 +407,7 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return
-        r = cpu_oracle_rate()
+        r = cpu_oracle_steps(args.steps, args.warmup)
         print(json.dumps({"impl": "reference", "metric": METRIC, "value": r["value"], "unit": "Gelem/s",
                           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
                           "ms_per_step": r["ms_per_step"], "higher_is_better": True, "scaling": "weak",
@@ -412,6 +481,9 @@ def main():
         "gpu_launches": len(VARIANTS) * args.steps,
         "clocks": clk.summary(),
     }
+    if not args.no_extras:
+        el = elements_mode(sb, dev, world, rank)
+        res["elements_mode_sharded_problem"] = el
     if rank == 0 and not args.no_e2e:
         res["e2e"] = e2e(sb)
     if rank == 0 and world == 1 and not args.no_cpu:
