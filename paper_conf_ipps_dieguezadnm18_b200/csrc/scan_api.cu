@@ -58,7 +58,7 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
 }
 int choose_lookback_variant(int64_t N, int64_t G) {
     const int64_t total = N * G;
-    if (N < 1024 && G > 1) return 3;
+    if (N < 1024 && G > 1) return 2;
     return total >= (int64_t(1) << 22) ? 0 : 1;
 }
 

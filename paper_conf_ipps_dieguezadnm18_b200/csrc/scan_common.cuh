@@ -411,6 +411,19 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
         " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
         " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(phase) : "memory");
 }
+// wait for an mbarrier phase, or give up once the stream's end index (published in shared
+// memory by the role that met the end sentinel) is < i; returns false in that case.  The
+// warp that owns the sentinel index itself (end == i) must wait: it forwards the sentinel.
+__device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t phase, const int64_t* end, int64_t i) {
+    while (true) {
+        uint32_t ok;
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(ok) : "r"(smem_u32(bar)), "r"(phase) : "memory");
+        if (ok) return true;
+        if (*(const volatile int64_t*)end < i) return false;
+    }
+}
 __device__ __forceinline__ uint4 lds_v4(const void* p) {
     uint4 r;
     asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)

@@ -100,7 +100,8 @@ struct Desc {
 // distance l + 32 m); it waits only for the predecessors up to the nearest inclusive (P)
 // one, folds their values and stops there, or slides the window further back.
 template <class Op, int M = LB_M>
-__device__ __forceinline__ typename Op::Carry look_back(const LookbackParams& p, int64_t t, uint32_t tag) {
+__device__ __forceinline__ typename Op::Carry look_back(const LookbackParams& p, int64_t t, uint32_t tag,
+                                                        uint32_t* stats = nullptr) {
     using C = typename Op::Carry;
     const int lane = lane_id();
     C run = Op::cidentity();
@@ -110,7 +111,9 @@ __device__ __forceinline__ typename Op::Carry look_back(const LookbackParams& p,
         uint32_t st[M];
         int dP;
         int spins = 0;
+        if (stats) stats[1] += 1;           // windows visited
         while (true) {
+            if (stats) stats[0] += 1;       // descriptor read round trips
 #pragma unroll
             for (int m = 0; m < M; ++m) {
                 const int64_t pred = front - lane - 32 * m;
@@ -148,8 +151,11 @@ __device__ __forceinline__ void trace_stamp(const LookbackParams& p, int64_t t, 
     if (p.trace != nullptr && t < p.trace_tiles) {
         uint64_t g;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
-        p.trace[4 * t + e] = g;
+        p.trace[8 * t + e] = g;
     }
+}
+__device__ __forceinline__ void trace_value(const LookbackParams& p, int64_t t, int e, uint64_t v) {
+    if (p.trace != nullptr && t < p.trace_tiles) p.trace[8 * t + e] = v;
 }
 
 __device__ __forceinline__ void consumer_bar(int nthreads) {
@@ -356,6 +362,7 @@ struct PipeCtx {
     uint64_t* p1;
     uint64_t* cr;
     uint64_t* empty;
+    int64_t* end;           // sequence index of the end sentinel (INT64_MAX until met)
 };
 
 // consumer: pass 1 of the tile in sequence slot i; false at the end sentinel
@@ -374,7 +381,10 @@ __device__ __forceinline__ bool pipe_pass1(const LookbackParams& p, const PipeCt
     mbar_wait(&c.full[slot], ph);
     SlotHdr<Op, WARPS>& h = c.hdr[slot];
     if (h.tid < 0) {
-        if (warp == WARPS - 1 && lane == 0) mbar_arrive(&c.p1[slot]);
+        if (warp == WARPS - 1 && lane == 0) {
+            *(volatile int64_t*)c.end = i;       // look-back warps waiting beyond i leave
+            mbar_arrive(&c.p1[slot]);
+        }
         return false;
     }
     if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 0);
@@ -440,8 +450,8 @@ __device__ __forceinline__ void pipe_pass2(const LookbackParams& p, const PipeCt
     if (lane == 0) mbar_arrive(&c.empty[slot]);
 }
 
-template <class Op, int WARPS, int V, int S, int M>
-__global__ void __launch_bounds__((WARPS + 2) * 32) lookback_pipelined_kernel(LookbackParams p, int64_t num_tiles) {
+template <class Op, int WARPS, int V, int S, int M, int NLB>
+__global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_kernel(LookbackParams p, int64_t num_tiles) {
     using T = typename Op::T;
     using C = typename Op::Carry;
     using Ctx = PipeCtx<Op, WARPS, V, S>;
@@ -450,10 +460,12 @@ __global__ void __launch_bounds__((WARPS + 2) * 32) lookback_pipelined_kernel(Lo
     __shared__ SlotHdr<Op, WARPS> s_hdr[S];
     __shared__ uint64_t s_full[S], s_p1[S], s_cr[S], s_empty[S];
     __shared__ uint32_t s_tag;
+    __shared__ int64_t s_end;
     const int warp = threadIdx.x >> 5, lane = lane_id();
-    Ctx c{(T*)dsm, s_hdr, s_full, s_p1, s_cr, s_empty};
+    Ctx c{(T*)dsm, s_hdr, s_full, s_p1, s_cr, s_empty, &s_end};
 
     if (threadIdx.x == 0) {
+        s_end = INT64_MAX;
 #pragma unroll
         for (int s = 0; s < S; ++s) {
             mbar_init(&s_full[s], 1); mbar_init(&s_p1[s], 1);
@@ -512,11 +524,13 @@ __global__ void __launch_bounds__((WARPS + 2) * 32) lookback_pipelined_kernel(Lo
             }
         }
     } else {
-        // ---------------- look-back warp: warp prefixes, publish, look back, carry
-        for (int64_t i = 0;; ++i) {
+        // ---------------- NLB look-back warps (tile sequence i -> warp i mod NLB); p1 phases
+        // complete in sequence order, so NLB <= S keeps every wait on the right phase
+        static_assert(NLB <= S, "look-back warps must not lap the ring");
+        for (int64_t i = warp - (WARPS + 1);; i += NLB) {
             const int slot = (int)(i % S);
             const uint32_t ph = (uint32_t)((i / S) & 1);
-            mbar_wait(&s_p1[slot], ph);
+            if (!mbar_wait_or_end(&s_p1[slot], ph, &s_end, i)) break;
             SlotHdr<Op, WARPS>& h = s_hdr[slot];
             const int64_t t = h.tid;
             if (t < 0) break;
@@ -524,11 +538,15 @@ __global__ void __launch_bounds__((WARPS + 2) * 32) lookback_pipelined_kernel(Lo
             const bool has_head = h.has_head != 0u;
             const C aggc = h.agg;
             C carry = Op::cidentity();
-            if (!starts) carry = look_back<Op, M>(p, t, tag);
+            uint32_t stats[2] = {0u, 0u};
+            if (lane == 0) trace_stamp(p, t, 4);
+            if (!starts) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
             if (lane == 0) {
                 if (!has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, aggc));
                 h.carry = carry;
                 trace_stamp(p, t, 2);
+                trace_value(p, t, 5, stats[0]);
+                trace_value(p, t, 6, stats[1]);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&s_cr[slot]);
@@ -564,20 +582,6 @@ __device__ __forceinline__ typename Op::T warp_reduce_rows(const typename Op::T*
 #pragma unroll
     for (int d = 16; d >= 1; d >>= 1) acc = Op::apply(acc, from_bits<T>(__shfl_xor_sync(FULL, to_bits<T>(acc), d)));
     return acc;
-}
-
-// wait for an mbarrier phase, or give up once the end index (set by the reducers when they
-// meet the end sentinel) is < i; returns false in the latter case.  The warp that owns the
-// sentinel index itself (end == i) must wait: it forwards the sentinel to P2.
-__device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t phase, const int64_t* end, int64_t i) {
-    while (true) {
-        uint32_t ok;
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(ok) : "r"(smem_u32(bar)), "r"(phase) : "memory");
-        if (ok) return true;
-        if (*(const volatile int64_t*)end < i) return false;
-    }
 }
 
 template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
@@ -903,12 +907,12 @@ cudaError_t launch_tma(const LookbackParams& p, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-template <class Op, int WARPS, int V, int S, int M>
+template <class Op, int WARPS, int V, int S, int M, int NLB>
 cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
     constexpr int SMEM = S * TILE * 4;
-    constexpr int THREADS = (WARPS + 2) * 32;
-    auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M>;
+    constexpr int THREADS = (WARPS + 1 + NLB) * 32;
+    auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M, NLB>;
     static int occ = 0;
     if (occ == 0) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
@@ -930,17 +934,20 @@ cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
 template <class Op>
 cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     switch (variant) {
-    case 0: return launch_pipelined<Op, 16, 8, 3, 5>(p, s);     // 16384-element tiles (64 KiB), window 160
-    case 1: return launch_pipelined<Op, 8, 8, 3, 4>(p, s);      // 8192-element tiles, 3 x 32 KiB ring
-    case 2: return launch_l2<Op, 8, 4, 3, 3, 32, 4, 4>(p, s);   // two reads (L2-staged), 8192-element tiles
-    default: return launch_tma<Op, 8, 8>(p, s);                 // one 8192-element tile per CTA
+    case 0: return launch_pipelined<Op, 16, 8, 3, 5, 1>(p, s);  // 16384-element tiles (64 KiB), window 160
+    case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1>(p, s);   // 8192-element tiles, 3 x 32 KiB ring
+    case 2: return launch_tma<Op, 8, 8>(p, s);                  // one 8192-element tile per CTA
+    case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);  // two reads (L2-staged), window 320 = 2 rounds
+    default: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s); // as 0 with two look-back warps
     }
 }
 
 }  // namespace
 
-int64_t lookback_tile_elems(int variant) { return variant == 0 ? 16384 : 8192; }
-int lookback_num_variants() { return 4; }
+int64_t lookback_tile_elems(int variant) {
+    return (variant == 0 || variant == 4) ? 16384 : 8192;
+}
+int lookback_num_variants() { return 5; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

@@ -1,5 +1,6 @@
-"""Timeline of the pipelined look-back kernel (scan_debug_trace): per-tile stamps
-0 data ready, 1 aggregate published, 2 inclusive published, 3 outputs written."""
+"""Timeline of the look-back kernels (scan_debug_trace), 8 u64 per tile:
+stamps 0 data ready, 1 aggregate published, 2 inclusive published, 3 outputs written,
+4 look-back started; counters 5 descriptor read round trips, 6 windows visited."""
 import argparse
 import os
 import sys
@@ -17,44 +18,49 @@ ap.add_argument("--dtype", default="i32")
 ap.add_argument("--G", type=int, default=1)
 ap.add_argument("--N", type=int, default=1 << 28)
 ap.add_argument("--param", type=int, default=0)
+ap.add_argument("--tile", type=int, default=0, help="tile elements (default: from the variant)")
 a = ap.parse_args()
 dt = {"i32": torch.int32, "f32": torch.float32}[a.dtype]
 x = torch.empty(a.G * a.N, dtype=torch.int32, device="cuda")
 inputs.fill_device(x, {"i32": "i32", "f32": "f32u"}[a.dtype], 7)
 x = x.view(dt).view(a.G, a.N)
 y = torch.empty_like(x)
-TILE = 16384 if a.param == 1 else 8192
+TILE = a.tile or {0: 16384, 4: 16384}.get(a.param, 8192)
 tiles = (a.G * a.N + TILE - 1) // TILE
-tr = torch.zeros(tiles * 4, dtype=torch.int64, device="cuda")
+tr = torch.zeros(tiles * 8, dtype=torch.int64, device="cuda")
 for _ in range(3):
     sb.scan(x, "add", out=y, algo="lookback", param=a.param)
 _lib.lib.scan_debug_trace(tr.data_ptr(), tiles)
 sb.scan(x, "add", out=y, algo="lookback", param=a.param)
 torch.cuda.synchronize()
 _lib.lib.scan_debug_trace(None, 0)
-T = tr.cpu().numpy().reshape(tiles, 4).astype(np.int64)
+R = tr.cpu().numpy().reshape(tiles, 8).astype(np.int64)
+T = R[:, :5].copy()
 T = T - T[:, 0].min()
-ok = (T[:, 0] >= 0) & (T[:, 3] > 0)
-print("tiles", tiles, "stamped", int(ok.sum()), "span us %.1f" % (T[:, 3].max() / 1e3))
+print("tiles", tiles, "span us %.1f" % (T[:, 3].max() / 1e3))
 
 
-def pct(v, name):
-    v = np.asarray(v, dtype=np.float64) / 1e3
-    print("%-28s p10 %7.2f  p50 %7.2f  p90 %7.2f  p99 %7.2f  mean %7.2f us" % (
-        name, *np.percentile(v, [10, 50, 90, 99]), v.mean()))
+def pct(v, name, scale=1e3, unit="us"):
+    v = np.asarray(v, dtype=np.float64) / scale
+    print("%-30s p10 %7.2f  p50 %7.2f  p90 %7.2f  p99 %7.2f  mean %7.2f %s" % (
+        name, *np.percentile(v, [10, 50, 90, 99]), v.mean(), unit))
 
 
 pct(T[:, 1] - T[:, 0], "ready -> A (pass1)")
-pct(T[:, 2] - T[:, 1], "A -> P (look-back)")
+pct(T[:, 4] - T[:, 1], "A -> look-back start (queue)")
+pct(T[:, 2] - T[:, 4], "look-back duration")
 pct(T[:, 3] - T[:, 2], "P -> written (pass2)")
 pct(T[:, 3] - T[:, 0], "ready -> written")
-for grid in (296, 148) if TILE == 8192 else (148,):
-    if tiles > 2 * grid:
-        cyc = T[grid:, 0] - T[:-grid, 0]
-        pct(cyc, "per-CTA cycle (grid %d)" % grid)
-pct(np.maximum(T[1:, 1], T[:-1, 2]) - T[1:, 1], "wait on pred P after own A")
-pct(T[1:, 2] - T[:-1, 2], "P(t) - P(t-1)")
-# front: P publish time vs tile index
-for q in (0.1, 0.25, 0.5, 0.75, 0.9, 1.0):
-    k = int(q * (tiles - 1))
-    print("tile %8d  ready %8.1f  A %8.1f  P %8.1f  done %8.1f us" % (k, *(T[k] / 1e3)))
+pct(R[:, 5], "descriptor round trips", 1, "")
+pct(R[:, 6], "windows", 1, "")
+lb = (T[:, 2] - T[:, 4]) / np.maximum(R[:, 5], 1)
+pct(lb, "look-back time / round trip")
+grid = 148 if TILE >= 16384 else 296
+if tiles > 2 * grid:
+    pct(T[grid:, 0] - T[:-grid, 0], "per-CTA cycle (grid %d)" % grid)
+nr = tiles // grid
+if nr > 2:
+    rr = T[: nr * grid, 0].reshape(nr, grid)
+    pct(rr.max(1) - rr.min(1), "data-ready spread per round")
+    pa = T[: nr * grid, 1].reshape(nr, grid)
+    pct(pa.max(1) - pa.min(1), "A spread per round")
