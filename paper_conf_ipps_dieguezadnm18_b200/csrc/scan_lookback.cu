@@ -445,6 +445,9 @@ __device__ __forceinline__ void pipe_pass2(const LookbackParams& p, const PipeCt
     const bool wpf = h.wpf[warp] != 0u;
     if (h.seg) st.template pass2<true>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
     else       st.template pass2<false>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+    // every lane's smem reads of this slot are ordered before lane 0's release-arrive on
+    // `empty`; the producer's acquire-wait on it precedes any rewrite of the slot
+    __threadfence_block();
     __syncwarp();
     if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 3);
     if (lane == 0) mbar_arrive(&c.empty[slot]);

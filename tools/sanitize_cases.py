@@ -1,0 +1,34 @@
+"""Small cases of every kernel family / variant for compute-sanitizer runs (T7).
+
+    compute-sanitizer --tool racecheck python tools/sanitize_cases.py [--quick]
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import inputs  # noqa: E402
+import paper_conf_ipps_dieguezadnm18_b200 as sb  # noqa: E402
+from paper_conf_ipps_dieguezadnm18_b200 import _lib  # noqa: E402
+
+quick = "--quick" in sys.argv
+shapes = [(20000, 3), (70001, 1), (1000, 40)] if not quick else [(70001, 1), (1000, 5)]
+cases = [("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0)] + \
+        [("lookback", v) for v in range(_lib.lib_num_lookback_variants())]
+for dt, dist in (("i32", "i32"), ("f32", "f32s")):
+    for N, G in shapes:
+        x = torch.empty(N * G, dtype=torch.int32, device="cuda")
+        inputs.fill_device(x, dist, 1)
+        if dt == "f32":
+            x = x.view(torch.float32)
+        x = x.view(G, N)
+        for algo, param in cases:
+            for kind in ("inclusive", "exclusive"):
+                sb.scan(x, "add", kind, algo=algo, param=param)
+                torch.cuda.synchronize()
+        t = sb.shard_totals(x, "add")
+        sb.shard_scan(x, torch.stack([t, t]), 1, 2, "add", "inclusive")
+        torch.cuda.synchronize()
+        print("ok", dt, N, G, flush=True)
+print("sanitize cases done")
