@@ -68,7 +68,7 @@ lib = _load()
 
 
 def lib_num_lookback_variants() -> int:
-    return 5
+    return 6
 
 
 def check(fn: str, code: int) -> None:

@@ -14,19 +14,25 @@
 // carry crosses problems.  Small N costs no extra launches and rows need not be 16-byte
 // aligned (only the base pointers).
 //
-// B200 structure (variants 0-2, persistent + warp-specialised):
-//   * one producer warp per CTA takes tile tickets (atomic, so tiles are handed out in
-//     start order: every tile waited on is owned by a running CTA) and streams the tiles
-//     into an S-stage shared-memory ring with 1-D TMA bulk copies (cp.async.bulk, SASS
-//     UBLKCP) completing on mbarriers -- the bytes in flight are bounded by smem, not by
-//     registers;
-//   * WARPS consumer warps scan each staged tile in two passes over smem (pass 1 prefixes,
-//     look-back by the last warp, pass 2 outputs with 128-bit streaming stores) and free
-//     the stage through an "empty" mbarrier;
-//   * the look-back window is 32*M tiles wide (each lane inspects M descriptors per
-//     round trip): a single huge problem (configs[2], N = 2^30) advances its inclusive
-//     front by up to 128 tiles per L2 round trip instead of 32.
-// Variant 3 is a non-persistent one-tile-per-CTA TMA kernel, kept for comparison.
+// B200 structure of the default kernel (variant 0, lookback_pipelined_kernel):
+//   * persistent, one CTA per SM; tiles of 16384 elements (64 KiB) are assigned round robin
+//     (tile = cta + k * grid; blocks dispatch in index order, so every tile a CTA waits on
+//     belongs to a CTA that is already running);
+//   * a producer warp streams the CTA's tiles into a 3-stage shared-memory ring with 1-D
+//     TMA bulk copies (cp.async.bulk, SASS UBLKCP) completing on mbarriers -- the bytes in
+//     flight are bounded by shared memory, not by registers;
+//   * 16 consumer warps scan each staged tile in two passes over smem; right after pass 1
+//     the last consumer warp publishes the tile aggregate (A), so aggregates never wait for
+//     a look-back; consumers run pass 1 of tile i+1 before pass 2 of tile i;
+//   * a dedicated look-back warp resolves each tile's carry with a 160-tile window (M = 5
+//     descriptors per lane per round trip, one window >= one round of 148 tiles).
+// Measured limits (tools/trace_lookback.py): a descriptor round trip costs
+// ~2 us under full HBM load and a tile holds its smem slot from TMA issue to pass 2, so a
+// single 2^30-element problem runs at ~80 % of the measured copy bandwidth.
+// Other variants (kept measurable through scan_batch_ex `param`): 1 = 32 KiB tiles,
+// 2 = one tile per CTA (short / unaligned rows), 3 = L2-staged two-read form (limited by
+// L2 slice throughput on B200), 4 = two look-back warps, 5 = register-resident waiting
+// tiles.
 //
 // Descriptors (one per tile; reset-free thanks to a 30-bit epoch tag in every word):
 //   word = payload32 << 32 | tag << 2 | status      status 0 X (not ready), 1 A, 2 P
@@ -559,6 +565,198 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
     if (threadIdx.x == 0) epilogue(p);
 }
 
+// ---------------------------------------------------------------- register-resident pipeline
+// As the pipelined kernel, but pass 1 leaves each element's warp-local prefix in registers
+// (WarpTileR) and releases the shared-memory slot at once: smem only covers load + pass 1,
+// and the tiles waiting for their carry sit in the register file (two per consumer warp).
+// Per-tile headers live in their own ring (SH entries) released after the outputs are
+// written.  Roles: WARPS consumers | producer (TMA) | look-back warp.
+template <class Op, int WARPS, int V, int S, int SH, int M>
+__global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(LookbackParams p, int64_t num_tiles) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int WCH = V * 128, TILE = WARPS * WCH;
+    extern __shared__ __align__(128) unsigned char dsm[];
+    T* data = (T*)dsm;
+    __shared__ SlotHdr<Op, WARPS> s_hdr[SH];
+    __shared__ uint64_t fullR[S], emptyR[S], p1[SH], cr[SH], emptyH[SH];
+    __shared__ uint32_t s_tag;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) { mbar_init(&fullR[s], 1); mbar_init(&emptyR[s], WARPS); }
+        for (int s = 0; s < SH; ++s) { mbar_init(&p1[s], 1); mbar_init(&cr[s], 1); mbar_init(&emptyH[s], WARPS); }
+        fence_mbar_init();
+        s_tag = read_tag(p);
+    }
+    __syncthreads();
+    const uint32_t tag = s_tag;
+    const bool excl = p.exclusive;
+
+    if (warp < WARPS) {
+        // ---------------- consumers
+        WarpTileR<Op, V> A, B;
+        auto pass1 = [&](WarpTileR<Op, V>& st, int64_t i) -> bool {
+            const int sR = (int)(i % S), sH = (int)(i % SH);
+            mbar_wait(&fullR[sR], (uint32_t)((i / S) & 1));
+            SlotHdr<Op, WARPS>& h = s_hdr[sH];
+            if (h.tid < 0) {
+                if (warp == WARPS - 1 && lane == 0) mbar_arrive(&p1[sH]);
+                return false;
+            }
+            if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 0);
+            const T* srow = data + (size_t)sR * TILE + warp * WCH;
+            const int64_t r = h.r;
+            if (h.seg) {
+                const bool small = p.N < TILE;
+                const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+                if (excl) st.template pass1<true, true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+                else      st.template pass1<true, false>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+            } else {
+                if (excl) st.template pass1<false, true>(srow, warp * WCH, false, 0u, 1u, -1);
+                else      st.template pass1<false, false>(srow, warp * WCH, false, 0u, 1u, -1);
+            }
+            __threadfence_block();
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&emptyR[sR]);                 // the tile now lives in registers
+                h.wtot[warp] = st.wtot;
+                h.wfl[warp] = st.wfl ? 1u : 0u;
+            }
+            consumer_bar(WARPS * 32);
+            if (warp == WARPS - 1) {
+                const bool seg = h.seg != 0u;
+                T run = Op::identity(); bool f = false;
+#pragma unroll
+                for (int w = 0; w < WARPS; ++w) {
+                    if (lane == w) { h.wp[w] = run; h.wpf[w] = f ? 1u : 0u; }
+                    const T v = h.wtot[w];
+                    const bool fw = seg && h.wfl[w] != 0u;
+                    run = fw ? v : Op::apply(run, v);
+                    f = f || fw;
+                }
+                const bool has_head = seg ? f : (r == 0);
+                if (lane == 0) {
+                    h.agg = Op::to_carry(run);
+                    h.has_head = has_head ? 1u : 0u;
+                    trace_stamp(p, h.tid, 1);
+                    Desc<Op>::publish(p, h.tid, tag, has_head ? ST_P : ST_A, h.agg);
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&p1[sH]);
+            }
+            return true;
+        };
+        auto pass2 = [&](const WarpTileR<Op, V>& st, int64_t i) {
+            const int sH = (int)(i % SH);
+            mbar_wait(&cr[sH], (uint32_t)((i / SH) & 1));
+            const SlotHdr<Op, WARPS>& h = s_hdr[sH];
+            const int64_t gidx = h.tid * (int64_t)TILE + warp * WCH;
+            const T cin = Op::from_carry(h.carry);
+            const T wp = h.wp[warp];
+            const bool wpf = h.wpf[warp] != 0u, fast = h.fast != 0u;
+            if (h.seg) st.template emit<true>((T*)p.out, gidx, p.total, fast, p.vec, wp, wpf, cin);
+            else       st.template emit<false>((T*)p.out, gidx, p.total, fast, p.vec, wp, wpf, cin);
+            __syncwarp();
+            if (lane == 0) {
+                if (warp == 0) trace_stamp(p, h.tid, 3);
+                mbar_arrive(&emptyH[sH]);
+            }
+        };
+        int64_t i = 0;
+        if (pass1(A, 0)) {
+            while (true) {
+                ++i;
+                bool more = pass1(B, i);
+                pass2(A, i - 1);
+                if (!more) break;
+                ++i;
+                more = pass1(A, i);
+                pass2(B, i - 1);
+                if (!more) break;
+            }
+        }
+    } else if (warp == WARPS) {
+        // ---------------- producer: this CTA's tiles (round robin) into the TMA ring
+        const T* in = (const T*)p.in;
+        const uint64_t pol = l2_evict_first_policy();
+        int64_t i = 0;
+        for (int64_t t = blockIdx.x;; t += gridDim.x, ++i) {
+            const int sR = (int)(i % S), sH = (int)(i % SH);
+            mbar_wait(&emptyR[sR], (uint32_t)((i / S) & 1) ^ 1u);
+            mbar_wait(&emptyH[sH], (uint32_t)((i / SH) & 1) ^ 1u);
+            SlotHdr<Op, WARPS>& h = s_hdr[sH];
+            if (t >= num_tiles) {
+                if (lane == 0) { h.tid = -1; mbar_arrive(&fullR[sR]); }
+                break;
+            }
+            const TileInfo ti = classify(p, t, TILE);
+            T* dst = data + (size_t)sR * TILE;
+            const int64_t base = t * (int64_t)TILE;
+            if (lane == 0) { h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast; }
+            if (ti.fast) {
+                if (lane == 0) {
+                    mbar_expect_tx(&fullR[sR], TILE * 4);
+                    tma_load_1d(dst, in + base, TILE * 4, &fullR[sR], pol);
+                }
+            } else {
+                for (int k = lane; k < TILE; k += 32)
+                    dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&fullR[sR]);
+            }
+        }
+    } else {
+        // ---------------- look-back warp
+        for (int64_t i = 0;; ++i) {
+            const int sH = (int)(i % SH);
+            mbar_wait(&p1[sH], (uint32_t)((i / SH) & 1));
+            SlotHdr<Op, WARPS>& h = s_hdr[sH];
+            const int64_t t = h.tid;
+            if (t < 0) break;
+            C carry = Op::cidentity();
+            uint32_t stats[2] = {0u, 0u};
+            if (lane == 0) trace_stamp(p, t, 4);
+            if (h.r != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            if (lane == 0) {
+                if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
+                h.carry = carry;
+                trace_stamp(p, t, 2);
+                trace_value(p, t, 5, stats[0]);
+                trace_value(p, t, 6, stats[1]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&cr[sH]);
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
+template <class Op, int WARPS, int V, int S, int SH, int M>
+cudaError_t launch_regs(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = WARPS * V * 128;
+    constexpr int SMEM = S * TILE * 4;
+    constexpr int THREADS = (WARPS + 2) * 32;
+    auto kern = lookback_regs_kernel<Op, WARPS, V, S, SH, M>;
+    static int occ = 0;
+    if (occ == 0) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        if (e != cudaSuccess) return e;
+        int o = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
+        if (e != cudaSuccess) return e;
+        if (o < 1) return cudaErrorInvalidConfiguration;
+        occ = o;
+    }
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    int64_t grid = (int64_t)occ * num_sms();
+    if (grid > tiles) grid = tiles;
+    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- two reads, L2-staged (variant 0)
 // Little's law: a tile that waits in shared memory for its carry holds a slot for the
 // whole look-back latency (several us under full HBM load), which caps a single huge
@@ -769,11 +967,15 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                 break;
             }
             C carry = Op::cidentity();
-            if (h.r != 0) carry = look_back<Op, M>(p, t, tag);
+            uint32_t stats[2] = {0u, 0u};
+            if (lane == 0) trace_stamp(p, t, 4);
+            if (h.r != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
             if (lane == 0) {
                 if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
                 h.carry = carry;
                 trace_stamp(p, t, 2);
+                trace_value(p, t, 5, stats[0]);
+                trace_value(p, t, 6, stats[1]);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&crd[sH]);
@@ -941,16 +1143,17 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1>(p, s);   // 8192-element tiles, 3 x 32 KiB ring
     case 2: return launch_tma<Op, 8, 8>(p, s);                  // one 8192-element tile per CTA
     case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);  // two reads (L2-staged), window 320 = 2 rounds
-    default: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s); // as 0 with two look-back warps
+    case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s);  // as 0 with two look-back warps
+    default: return launch_regs<Op, 12, 8, 4, 8, 5>(p, s);      // register-resident waiting tiles, 48 KiB
     }
 }
 
 }  // namespace
 
 int64_t lookback_tile_elems(int variant) {
-    return (variant == 0 || variant == 4) ? 16384 : 8192;
+    return (variant == 0 || variant == 4) ? 16384 : variant == 5 ? 12288 : 8192;
 }
-int lookback_num_variants() { return 5; }
+int lookback_num_variants() { return 6; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

@@ -25,7 +25,7 @@ x = torch.empty(a.G * a.N, dtype=torch.int32, device="cuda")
 inputs.fill_device(x, {"i32": "i32", "f32": "f32u"}[a.dtype], 7)
 x = x.view(dt).view(a.G, a.N)
 y = torch.empty_like(x)
-TILE = a.tile or {0: 16384, 4: 16384}.get(a.param, 8192)
+TILE = a.tile or {0: 16384, 4: 16384, 5: 12288}.get(a.param, 8192)
 tiles = (a.G * a.N + TILE - 1) // TILE
 tr = torch.zeros(tiles * 8, dtype=torch.int64, device="cuda")
 for _ in range(3):
@@ -55,7 +55,7 @@ pct(R[:, 5], "descriptor round trips", 1, "")
 pct(R[:, 6], "windows", 1, "")
 lb = (T[:, 2] - T[:, 4]) / np.maximum(R[:, 5], 1)
 pct(lb, "look-back time / round trip")
-grid = 148 if TILE >= 16384 else 296
+grid = 148 if (TILE >= 12288 or a.param == 3) else 296
 if tiles > 2 * grid:
     pct(T[grid:, 0] - T[:-grid, 0], "per-CTA cycle (grid %d)" % grid)
 nr = tiles // grid
