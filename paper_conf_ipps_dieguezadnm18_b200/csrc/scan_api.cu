@@ -247,14 +247,31 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
 // Three streams per device: copy-in, compute, copy-out; S staging slots of kPiece
 // elements rotate through them so the H2D copy of unit u+1, the scan of unit u and the
 // D2H copy of unit u-1 overlap (both copy engines busy: PCIe is full duplex).
-constexpr int kSlots = 3;
-constexpr int64_t kPiece = int64_t(1) << 24;      // 64 MiB of 32-bit elements per slot
+// Staging granularity: small enough that the first copy-in and the last copy-out (which
+// cannot overlap anything) are short, large enough to amortise per-copy costs.  Defaults
+// from the on-box e2e sweep; SCANB200_HOST_PIECE / SCANB200_HOST_SLOTS override them.
+constexpr int kMaxSlots = 8;
+
+int64_t env_i64(const char* name, int64_t dflt, int64_t lo, int64_t hi) {
+    const char* s = std::getenv(name);
+    if (!s) return dflt;
+    const long long v = std::atoll(s);
+    return v < lo ? lo : v > hi ? hi : v;
+}
+int64_t host_piece() {                               // elements per staging slot
+    static const int64_t v = env_i64("SCANB200_HOST_PIECE", int64_t(1) << 22, int64_t(1) << 16, int64_t(1) << 26);
+    return v;
+}
+int host_slots() {
+    static const int v = (int)env_i64("SCANB200_HOST_SLOTS", 4, 2, kMaxSlots);
+    return v;
+}
 
 struct HostCtx {
     bool init = false;
     cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
-    void* slot[kSlots] = {};
-    cudaEvent_t ev_in[kSlots] = {}, ev_scan[kSlots] = {}, ev_out[kSlots] = {};
+    void* slot[kMaxSlots] = {};
+    cudaEvent_t ev_in[kMaxSlots] = {}, ev_scan[kMaxSlots] = {}, ev_out[kMaxSlots] = {};
     uint64_t* piece_totals = nullptr;
     int64_t piece_cap = 0;
 };
@@ -268,8 +285,8 @@ scan_status host_ctx(int dev, HostCtx** out) {
             cudaStreamCreateWithFlags(&c.comp, cudaStreamNonBlocking) != cudaSuccess ||
             cudaStreamCreateWithFlags(&c.d2h, cudaStreamNonBlocking) != cudaSuccess)
             return SCAN_ERR_CUDA;
-        for (int k = 0; k < kSlots; ++k) {
-            if (cudaMalloc(&c.slot[k], kPiece * 4) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
+        for (int k = 0; k < host_slots(); ++k) {
+            if (cudaMalloc(&c.slot[k], host_piece() * 4) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
             if (cudaEventCreateWithFlags(&c.ev_in[k], cudaEventDisableTiming) != cudaSuccess ||
                 cudaEventCreateWithFlags(&c.ev_scan[k], cudaEventDisableTiming) != cudaSuccess ||
                 cudaEventCreateWithFlags(&c.ev_out[k], cudaEventDisableTiming) != cudaSuccess)
@@ -289,6 +306,8 @@ scan_status host_pipeline(const void* in_host, void* out_host, int64_t N, int64_
     HostCtx* c = nullptr;
     scan_status st = host_ctx(dev, &c);
     if (st != SCAN_OK) return st;
+    const int64_t kPiece = host_piece();
+    const int kSlots = host_slots();
     const bool pieces = N > kPiece;
     const int64_t npieces = pieces ? (N + kPiece - 1) / kPiece : 0;
     if (pieces && c->piece_cap < npieces) {
