@@ -535,21 +535,24 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
     } else {
         // ---------------- NLB look-back warps (tile sequence i -> warp i mod NLB); p1 phases
         // complete in sequence order, so NLB <= S keeps every wait on the right phase
+        // The tile of sequence i is known statically (round robin), and a look-back reads
+        // only the tile's predecessors, so it starts BEFORE the tile's own pass 1 is done;
+        // only publishing P waits for this tile's aggregate (p1).
         static_assert(NLB <= S, "look-back warps must not lap the ring");
         for (int64_t i = warp - (WARPS + 1);; i += NLB) {
+            const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
+            if (t >= num_tiles) break;
             const int slot = (int)(i % S);
             const uint32_t ph = (uint32_t)((i / S) & 1);
-            if (!mbar_wait_or_end(&s_p1[slot], ph, &s_end, i)) break;
-            SlotHdr<Op, WARPS>& h = s_hdr[slot];
-            const int64_t t = h.tid;
-            if (t < 0) break;
-            const bool starts = (h.r == 0);
-            const bool has_head = h.has_head != 0u;
-            const C aggc = h.agg;
+            const bool starts = ((t * (int64_t)TILE) % p.N) == 0;
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
             if (lane == 0) trace_stamp(p, t, 4);
             if (!starts) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            mbar_wait(&s_p1[slot], ph);                   // this tile's aggregate is in the header
+            SlotHdr<Op, WARPS>& h = s_hdr[slot];
+            const bool has_head = h.has_head != 0u;
+            const C aggc = h.agg;
             if (lane == 0) {
                 if (!has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, aggc));
                 h.carry = carry;
@@ -1144,16 +1147,20 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 2: return launch_tma<Op, 8, 8>(p, s);                  // one 8192-element tile per CTA
     case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);  // two reads (L2-staged), window 320 = 2 rounds
     case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s);  // as 0 with two look-back warps
-    default: return launch_regs<Op, 12, 8, 4, 8, 5>(p, s);      // register-resident waiting tiles, 48 KiB
+    case 5: return launch_regs<Op, 12, 8, 4, 8, 5>(p, s);       // register-resident waiting tiles, 48 KiB
+    case 6: return launch_tma<Op, 8, 4>(p, s);                  // one 4096-element tile per CTA
+    case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);   // 4096-element tiles, 4 x 16 KiB ring
+    default: return launch_pipelined<Op, 18, 8, 3, 5, 1>(p, s); // 18432-element tiles (72 KiB), 216 KiB ring
     }
 }
 
 }  // namespace
 
 int64_t lookback_tile_elems(int variant) {
-    return (variant == 0 || variant == 4) ? 16384 : variant == 5 ? 12288 : 8192;
+    return (variant == 0 || variant == 4) ? 16384 : variant == 5 ? 12288 : variant == 8 ? 18432
+         : variant >= 6 ? 4096 : 8192;
 }
-int lookback_num_variants() { return 6; }
+int lookback_num_variants() { return 9; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

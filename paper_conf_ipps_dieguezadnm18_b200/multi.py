@@ -30,7 +30,7 @@ import torch.distributed as dist
 from . import _lib, shard_scan, shard_totals
 from ._lib import KINDS, OPS, check
 
-__all__ = ["partition", "exchange_totals", "scan_multi", "NativeComm"]
+__all__ = ["partition", "grouped_plan", "make_groups", "exchange_totals", "scan_multi", "NativeComm"]
 
 
 def partition(n: int, world: int, rank: int) -> tuple[int, int]:
@@ -43,6 +43,36 @@ def partition(n: int, world: int, rank: int) -> tuple[int, int]:
     if world < 1 or not 0 <= rank < world or n < 0:
         raise ValueError("bad partition arguments")
     return (rank * n) // world, ((rank + 1) * n) // world
+
+
+def grouped_plan(G: int, N: int, world: int, V: int, rank: int) -> dict:
+    """MP-PC-style grouping (PAPER.md:213-217 [§4.1.1, Fig. 8]): the W ranks form Y = W/V
+    groups of V consecutive ranks; group y solves problems [floor(yG/Y), floor((y+1)G/Y))
+    and, inside the group, rank v owns the contiguous portion v of each of those problems
+    (the paper's "V GPUs of each PCI-e network work on G/Y problems, partitioning each
+    problem into V portions of size N/V").  On NVSwitch the topology is uniform, so V only
+    trades exchange fan-in against per-problem parallelism."""
+    if V < 1 or world % V:
+        raise ValueError("V must divide the world size")
+    Y = world // V
+    y, v = divmod(rank, V)
+    g0, g1 = partition(G, Y, y)
+    e0, e1 = partition(N, V, v)
+    return {"groups": Y, "group": y, "member": v, "problems": (g0, g1), "elements": (e0, e1)}
+
+
+def make_groups(V: int):
+    """Create the Y = W/V sub-communicators of :func:`grouped_plan` (collective: every rank
+    calls it; every rank takes part in creating every group) and return this rank's."""
+    world, rank = dist.get_world_size(), dist.get_rank()
+    if V < 1 or world % V:
+        raise ValueError("V must divide the world size")
+    mine = None
+    for y in range(world // V):
+        g = dist.new_group(list(range(y * V, (y + 1) * V)))
+        if y == rank // V:
+            mine = g
+    return mine
 
 
 def exchange_totals(totals: torch.Tensor, group=None) -> torch.Tensor:
@@ -81,6 +111,8 @@ def scan_multi(x_local: torch.Tensor, op: str = "add", kind: str = "inclusive", 
 
     mode="problems": x_local holds whole problems (this rank's partition of the batch).
     mode="elements": x_local holds this rank's portion of each of the G problems.
+    MP-PC grouping = mode="elements" with ``group`` = this rank's sub-communicator from
+    :func:`make_groups` and x_local laid out by :func:`grouped_plan`.
     Collective in elements mode: every rank of ``group`` must call it with the same G,
     op, kind, mode and backend.
     """

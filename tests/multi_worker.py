@@ -65,3 +65,28 @@ def gloo_problems_worker(rank, world, port, G, result_dir):
     with open(os.path.join(result_dir, "rank%d" % rank), "w") as f:
         f.write("ok" if ok else "BAD %s" % spans)
     dist.destroy_process_group()
+
+
+def gloo_grouped_worker(rank, world, port, V, G, N, result_dir):
+    """MP-PC grouping: Y = W/V groups, each scatters its problems over its V ranks."""
+    _init(rank, world, port, "gloo")
+    from paper_conf_ipps_dieguezadnm18_b200.multi import exchange_totals, grouped_plan, make_groups
+    sub = make_groups(V)
+    plan = grouped_plan(G, N, world, V, rank)
+    g0, g1 = plan["problems"]
+    e0, e1 = plan["elements"]
+    full = inputs.generate("i32", G * N, 77).reshape(G, N)
+    xl = np.ascontiguousarray(full[g0:g1, e0:e1])
+    ng = g1 - g0
+    tot = oracle.totals(xl, N=e1 - e0) if (e1 > e0 and ng) else np.zeros(ng, np.uint32)
+    allt = exchange_totals(torch.from_numpy(tot.astype(np.int64)), group=sub)     # [V, ng]
+    v = plan["member"]
+    carry = (allt[:v].numpy().astype(np.uint64).sum(axis=0) & 0xFFFFFFFF).astype(np.uint32) if v \
+        else np.zeros(ng, np.uint32)
+    local = oracle.scan(xl, "add").view(np.uint32) if (e1 > e0 and ng) else np.zeros((ng, e1 - e0), np.uint32)
+    got = (local + carry[:, None]).view(np.int32)
+    ok = np.array_equal(got, oracle.scan(full, "add")[g0:g1, e0:e1])
+    with open(os.path.join(result_dir, "rank%d" % rank), "w") as f:
+        f.write("ok" if ok else "BAD")
+    dist.barrier()
+    dist.destroy_process_group()

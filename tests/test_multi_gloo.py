@@ -40,3 +40,23 @@ def test_gloo_problems_mode(tmp_path):
     mp.spawn(multi_worker.gloo_problems_worker, args=(2, _port(), 4097, str(tmp_path)), nprocs=2, join=True)
     for r in range(2):
         assert open(os.path.join(tmp_path, "rank%d" % r)).read() == "ok"
+
+
+def test_grouped_plan_covers_everything():
+    from paper_conf_ipps_dieguezadnm18_b200.multi import grouped_plan
+    G, N, W, V = 7, 1001, 8, 4
+    cells = set()
+    for r in range(W):
+        p = grouped_plan(G, N, W, V, r)
+        assert p["groups"] == 2 and p["group"] == r // V and p["member"] == r % V
+        for g in range(*p["problems"]):
+            cells.add((g, p["elements"]))
+    for g in range(G):
+        spans = sorted(e for gg, e in cells if gg == g)
+        assert spans[0][0] == 0 and spans[-1][1] == N and len(spans) == V
+
+
+def test_gloo_grouped_mode(tmp_path):
+    mp.spawn(multi_worker.gloo_grouped_worker, args=(4, _port(), 2, 5, 3001, str(tmp_path)), nprocs=4, join=True)
+    for r in range(4):
+        assert open(os.path.join(tmp_path, "rank%d" % r)).read() == "ok"
