@@ -574,7 +574,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
 // and the tiles waiting for their carry sit in the register file (two per consumer warp).
 // Per-tile headers live in their own ring (SH entries) released after the outputs are
 // written.  Roles: WARPS consumers | producer (TMA) | look-back warp.
-template <class Op, int WARPS, int V, int S, int SH, int M>
+template <class Op, int WARPS, int V, int S, int SH, int M, int NST>
 __global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(LookbackParams p, int64_t num_tiles) {
     using T = typename Op::T;
     using C = typename Op::Carry;
@@ -666,6 +666,9 @@ __global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(Look
                 mbar_arrive(&emptyH[sH]);
             }
         };
+        // (a third register state would let consumers run two tiles ahead, but at 448
+        //  threads ptxas caps the kernel at 128 registers and it spills: measured slower)
+        static_assert(NST == 2, "two register states per consumer warp");
         int64_t i = 0;
         if (pass1(A, 0)) {
             while (true) {
@@ -710,17 +713,17 @@ __global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(Look
             }
         }
     } else {
-        // ---------------- look-back warp
+        // ---------------- look-back warp (speculative: starts before the tile's pass 1)
         for (int64_t i = 0;; ++i) {
+            const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
+            if (t >= num_tiles) break;
             const int sH = (int)(i % SH);
-            mbar_wait(&p1[sH], (uint32_t)((i / SH) & 1));
-            SlotHdr<Op, WARPS>& h = s_hdr[sH];
-            const int64_t t = h.tid;
-            if (t < 0) break;
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
             if (lane == 0) trace_stamp(p, t, 4);
-            if (h.r != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            if (((t * (int64_t)TILE) % p.N) != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            mbar_wait(&p1[sH], (uint32_t)((i / SH) & 1));
+            SlotHdr<Op, WARPS>& h = s_hdr[sH];
             if (lane == 0) {
                 if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
                 h.carry = carry;
@@ -736,12 +739,12 @@ __global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(Look
     if (threadIdx.x == 0) epilogue(p);
 }
 
-template <class Op, int WARPS, int V, int S, int SH, int M>
+template <class Op, int WARPS, int V, int S, int SH, int M, int NST>
 cudaError_t launch_regs(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * V * 128;
     constexpr int SMEM = S * TILE * 4;
     constexpr int THREADS = (WARPS + 2) * 32;
-    auto kern = lookback_regs_kernel<Op, WARPS, V, S, SH, M>;
+    auto kern = lookback_regs_kernel<Op, WARPS, V, S, SH, M, NST>;
     static int occ = 0;
     if (occ == 0) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
@@ -1147,7 +1150,7 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 2: return launch_tma<Op, 8, 8>(p, s);                  // one 8192-element tile per CTA
     case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);  // two reads (L2-staged), window 320 = 2 rounds
     case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s);  // as 0 with two look-back warps
-    case 5: return launch_regs<Op, 12, 8, 4, 8, 5>(p, s);       // register-resident waiting tiles, 48 KiB
+    case 5: return launch_regs<Op, 12, 8, 4, 8, 5, 2>(p, s);    // register-resident waiting tiles, 48 KiB
     case 6: return launch_tma<Op, 8, 4>(p, s);                  // one 4096-element tile per CTA
     case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);   // 4096-element tiles, 4 x 16 KiB ring
     default: return launch_pipelined<Op, 18, 8, 3, 5, 1>(p, s); // 18432-element tiles (72 KiB), 216 KiB ring
