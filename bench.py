@@ -326,12 +326,28 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         ms = float(t.item())
         comm.close()
+    # per-phase breakdown (the paper's Fig. 14): Stage 1+2 / exchange /
+    # Stage 3, events between the three steps of the torch-backend path
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+    ph = [0.0, 0.0, 0.0]
+    for _ in range(reps):
+        ev[0].record()
+        t = sb.shard_totals(x, "add")
+        ev[1].record()
+        allt = multi.exchange_totals(t) if world > 1 else t.view(1, -1)
+        ev[2].record()
+        sb.shard_scan(x, allt, rank, world, "add", "inclusive", out=y)
+        ev[3].record()
+        torch.cuda.synchronize()
+        for k in range(3):
+            ph[k] += ev[k].elapsed_time(ev[k + 1]) / reps
     hbm, _, _ = _peaks()
     per_gpu_gbs = 12.0 * n_local / (ms * 1e-3) / 1e9          # reduce pass (4 B) + scan pass (8 B)
     return {"N_total": world * n_local, "N_per_gpu": n_local, "ms": ms,
             "Gelem/s": world * n_local / ms / 1e6, "per_gpu_GB/s_at_12B_per_elem": per_gpu_gbs,
             "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
-            "exchange": "NCCL allgather (scan_batch_multi, native comm)" if world > 1 else "none (W=1)"}
+            "exchange": "NCCL allgather (scan_batch_multi, native comm)" if world > 1 else "none (W=1)",
+            "phases_ms_rank%d" % rank: {"stage1+2_reduce": ph[0], "exchange": ph[1], "stage3_scan": ph[2]}}
 
 
 def sweep(sb, dev):

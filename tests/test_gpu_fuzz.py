@@ -1,0 +1,39 @@
+"""Randomised parity: random shapes, ops, dtypes, kinds, kernel families, variants and
+pointer offsets (seeded), each checked element by element against the oracle."""
+import random
+
+import numpy as np
+import pytest
+import torch
+
+import inputs
+import paper_conf_ipps_dieguezadnm18_b200 as sb
+from gpu_util import COMBOS, DIST, NP, assert_parity, to_device, to_host
+from paper_conf_ipps_dieguezadnm18_b200 import _lib
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_cases(seed):
+    rng = random.Random(2018 + seed)
+    algos = [("auto", -1), ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0), ("three_stage", 3)] + \
+            [("lookback", v) for v in range(_lib.lib_num_lookback_variants())]
+    for case in range(40):
+        N = rng.choice([rng.randint(1, 300), rng.randint(300, 20000), rng.randint(20000, 400000)])
+        G = rng.choice([1, 1, 2, rng.randint(1, 40)])
+        if N * G > 3_000_000:
+            G = max(1, 3_000_000 // N)
+        op, dt = rng.choice(COMBOS)
+        kind = rng.choice(["inclusive", "exclusive"])
+        algo, param = rng.choice(algos)
+        off = rng.choice([0, 0, 1, 2, 3])
+        x = inputs.generate(DIST[dt], N * G + off, seed=seed * 1000 + case)
+        base = to_device(x)
+        xin = base[off: off + N * G].view(G, N)
+        out = torch.empty(N * G + 4, dtype=base.dtype, device="cuda")[off: off + N * G].view(G, N)
+        sb.scan(xin, op, kind, out=out, algo=algo, param=param)
+        torch.cuda.synchronize()
+        assert_parity(to_host(out, NP[dt]).reshape(G, N), x[off:].reshape(G, N), op, kind,
+                      label="fuzz seed=%d case=%d %s/%d %s %s %s N=%d G=%d off=%d" % (
+                          seed, case, algo, param, op, dt, kind, N, G, off))
