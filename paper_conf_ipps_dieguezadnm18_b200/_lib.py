@@ -68,7 +68,7 @@ lib = _load()
 
 
 def lib_num_lookback_variants() -> int:
-    return 9
+    return 10
 
 
 def check(fn: str, code: int) -> None:

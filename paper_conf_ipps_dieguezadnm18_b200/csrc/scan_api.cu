@@ -50,10 +50,14 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 //   few large problems (G*N >= 2^22): pipelined look-back with 64 KiB tiles;
 //   small totals (latency bound, L2 resident): pipelined look-back with 32 KiB tiles.
 // `aligned` = both base pointers 16-byte aligned.
+//   small totals of few problems (<= 2^22 elements, L2 resident, latency bound): the
+//     paper's three-stage form -- three short kernels beat one persistent look-back launch
+//     in device time (configs[0]: ~6 us vs ~7.5 us).
 scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
     if (rows_aligned && G >= 592 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
     if (rows_aligned && G >= 1184 && N >= 1024) return SCAN_ALGO_CASCADE_WARP;
+    if (G <= 16 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     return SCAN_ALGO_LOOKBACK;
 }
 int choose_lookback_variant(int64_t N, int64_t G) {
@@ -209,6 +213,9 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
                      cudaStream_t s) {
     if (algo == SCAN_ALGO_AUTO) {
         algo = choose_algo(N, G, (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0));
+        // a caller workspace is sized and laid out for the look-back family
+        // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage scratch into it
+        if (ws && algo == SCAN_ALGO_THREE_STAGE) algo = SCAN_ALGO_LOOKBACK;
         param = -1;
     }
     switch (algo) {

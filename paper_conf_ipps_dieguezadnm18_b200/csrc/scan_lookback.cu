@@ -459,7 +459,7 @@ __device__ __forceinline__ void pipe_pass2(const LookbackParams& p, const PipeCt
     if (lane == 0) mbar_arrive(&c.empty[slot]);
 }
 
-template <class Op, int WARPS, int V, int S, int M, int NLB>
+template <class Op, int WARPS, int V, int S, int M, int NLB, int PF = 0>
 __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_kernel(LookbackParams p, int64_t num_tiles) {
     using T = typename Op::T;
     using C = typename Op::Carry;
@@ -530,6 +530,17 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
                     dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&s_full[slot]);
+            }
+            if constexpr (PF > 0) {
+                // warm L2 with this CTA's tiles PF rounds ahead (first iteration: rounds 1..PF)
+                if (lane == 0 && p.vec) {
+#pragma unroll
+                    for (int r = (PF > 0 ? 1 : 0); r <= PF; ++r) {
+                        if (i > 0 && r < PF) continue;
+                        const int64_t tp = t + (int64_t)r * gridDim.x;
+                        if ((tp + 1) * (int64_t)TILE <= p.total) prefetch_l2_bulk(in + tp * (int64_t)TILE, TILE * 4);
+                    }
+                }
             }
         }
     } else {
@@ -1118,12 +1129,12 @@ cudaError_t launch_tma(const LookbackParams& p, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-template <class Op, int WARPS, int V, int S, int M, int NLB>
+template <class Op, int WARPS, int V, int S, int M, int NLB, int PF = 0>
 cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
     constexpr int SMEM = S * TILE * 4;
     constexpr int THREADS = (WARPS + 1 + NLB) * 32;
-    auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M, NLB>;
+    auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M, NLB, PF>;
     static int occ = 0;
     if (occ == 0) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
@@ -1145,25 +1156,26 @@ cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
 template <class Op>
 cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     switch (variant) {
-    case 0: return launch_pipelined<Op, 16, 8, 3, 5, 1>(p, s);  // 16384-element tiles (64 KiB), window 160
-    case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1>(p, s);   // 8192-element tiles, 3 x 32 KiB ring
-    case 2: return launch_tma<Op, 8, 8>(p, s);                  // one 8192-element tile per CTA
-    case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);  // two reads (L2-staged), window 320 = 2 rounds
-    case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2>(p, s);  // as 0 with two look-back warps
-    case 5: return launch_regs<Op, 12, 8, 4, 8, 5, 2>(p, s);    // register-resident waiting tiles, 48 KiB
-    case 6: return launch_tma<Op, 8, 4>(p, s);                  // one 4096-element tile per CTA
-    case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);   // 4096-element tiles, 4 x 16 KiB ring
-    default: return launch_pipelined<Op, 18, 8, 3, 5, 1>(p, s); // 18432-element tiles (72 KiB), 216 KiB ring
+    case 0: return launch_pipelined<Op, 16, 8, 3, 5, 1, 1>(p, s);  // 64 KiB tiles, window 160, L2 prefetch +1 round
+    case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1, 0>(p, s);   // 32 KiB tiles (small, L2-resident totals)
+    case 2: return launch_tma<Op, 8, 8>(p, s);                     // one 8192-element tile per CTA
+    case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);     // two reads (L2-staged), window 320 = 2 rounds
+    case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2, 1>(p, s);  // as 0 with two look-back warps
+    case 5: return launch_regs<Op, 12, 8, 4, 8, 5, 2>(p, s);       // register-resident waiting tiles, 48 KiB
+    case 6: return launch_tma<Op, 8, 4>(p, s);                     // one 4096-element tile per CTA
+    case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);      // 16 KiB tiles, 4-slot ring
+    case 8: return launch_pipelined<Op, 18, 8, 3, 5, 1, 2>(p, s);  // 72 KiB tiles, L2 prefetch +2 rounds
+    default: return launch_pipelined<Op, 16, 8, 3, 5, 1, 0>(p, s); // as 0 without the L2 prefetch
     }
 }
 
 }  // namespace
 
 int64_t lookback_tile_elems(int variant) {
-    return (variant == 0 || variant == 4) ? 16384 : variant == 5 ? 12288 : variant == 8 ? 18432
-         : variant >= 6 ? 4096 : 8192;
+    return (variant == 0 || variant == 4 || variant == 9) ? 16384 : variant == 5 ? 12288
+         : variant == 8 ? 18432 : (variant == 6 || variant == 7) ? 4096 : 8192;
 }
-int lookback_num_variants() { return 9; }
+int lookback_num_variants() { return 10; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

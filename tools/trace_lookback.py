@@ -25,7 +25,7 @@ x = torch.empty(a.G * a.N, dtype=torch.int32, device="cuda")
 inputs.fill_device(x, {"i32": "i32", "f32": "f32u"}[a.dtype], 7)
 x = x.view(dt).view(a.G, a.N)
 y = torch.empty_like(x)
-TILE = a.tile or {0: 16384, 4: 16384, 5: 12288}.get(a.param, 8192)
+TILE = a.tile or {0: 16384, 4: 16384, 9: 16384, 5: 12288, 8: 18432, 6: 4096, 7: 4096}.get(a.param, 8192)
 tiles = (a.G * a.N + TILE - 1) // TILE
 tr = torch.zeros(tiles * 8, dtype=torch.int64, device="cuda")
 for _ in range(3):
