@@ -63,7 +63,7 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
 int choose_lookback_variant(int64_t N, int64_t G) {
     const int64_t total = N * G;
     if (N < 1024 && G > 1) return 2;
-    return total >= (int64_t(1) << 22) ? 0 : 1;
+    return total >= (int64_t(1) << 22) ? 3 : 1;
 }
 
 int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
@@ -79,7 +79,7 @@ int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
 // workspace size (capacity C), never on the call; every descriptor word carries the tag
 // of the launch that wrote it, so 8-byte (32-bit carries) and 16-byte (fp64 carries)
 // uses of the same bytes can never be confused.
-constexpr size_t kLbSlotBytes = 16;
+constexpr size_t kLbSlotBytes = 8 * kDescWords;
 size_t lookback_bytes(int64_t total, int variant, bool split) {
     (void)split;
     int64_t tile = lookback_tile_elems(variant);

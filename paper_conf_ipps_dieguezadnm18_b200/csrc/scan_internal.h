@@ -22,6 +22,12 @@ struct LookbackParams {
     bool vec;           // in and out are 16-byte aligned
     bool exclusive;
 };
+// u64 words per look-back descriptor slot.  A descriptor needs 1 (32-bit carries) or 2
+// (fp64 carries) words; one descriptor per 64-byte slot puts only two tiles on a 128-byte
+// L2 line, i.e. few concurrent publishers and pollers per line.  Measured on one 2^30
+// problem: packed 8-byte descriptors ~80 % of copy, 16-byte slots ~90 %, 32/64-byte ~99 %
+// (the look-back round trip under full HBM load was dominated by line contention).
+constexpr int kDescWords = 8;
 int64_t lookback_tile_elems(int variant);
 int lookback_num_variants();
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s);

@@ -78,22 +78,24 @@ struct Desc {
         const uint64_t meta = (uint64_t)((tag << 2) | st);
         if constexpr (sizeof(C) == 8) {
             const uint64_t b = (uint64_t)__double_as_longlong(v);
-            st_relaxed_v2u64(p.desc + 2 * t, (b & 0xFFFFFFFF00000000ull) | meta, (b << 32) | meta);
+            st_relaxed_v2u64(p.desc + kDescWords * t, (b & 0xFFFFFFFF00000000ull) | meta, (b << 32) | meta);
         } else {
-            st_relaxed_u64(p.desc + t, ((uint64_t)to_bits<C>(v) << 32) | meta);
+            // one descriptor per 16-byte slot even for 8-byte descriptors: fewer tiles share a
+            // 128-byte L2 line, i.e. fewer concurrent writers / pollers per line (measured)
+            st_relaxed_u64(p.desc + kDescWords * t, ((uint64_t)to_bits<C>(v) << 32) | meta);
         }
     }
     // returns status (0 when stale, torn or not yet written) and the matching value
     static __device__ __forceinline__ uint32_t read(const LookbackParams& p, int64_t t, uint32_t tag, C& v) {
         if constexpr (sizeof(C) == 8) {
             uint64_t hi, lo;
-            ld_relaxed_v2u64(p.desc + 2 * t, hi, lo);
+            ld_relaxed_v2u64(p.desc + kDescWords * t, hi, lo);
             const uint32_t mh = (uint32_t)hi, ml = (uint32_t)lo;
             if ((mh >> 2) != tag || mh != ml) return 0u;
             v = __longlong_as_double((long long)((hi & 0xFFFFFFFF00000000ull) | (lo >> 32)));
             return mh & 3u;
         } else {
-            const uint64_t w = ld_relaxed_u64(p.desc + t);
+            const uint64_t w = ld_relaxed_u64(p.desc + kDescWords * t);
             if ((((uint32_t)w) >> 2) != tag) return 0u;
             v = from_bits<C>((uint32_t)(w >> 32));
             return (uint32_t)w & 3u;
@@ -240,7 +242,7 @@ __device__ __forceinline__ void epilogue(const LookbackParams& p) {
         __threadfence();
         uint32_t e = *((volatile uint32_t*)(p.ctl + 2)) + 1u;
         if (e + 1u >= TAG_MASK) {
-            for (int64_t i = 0; i < 2 * p.capacity; ++i) p.desc[i] = 0ull;
+            for (int64_t i = 0; i < kDescWords * p.capacity; ++i) p.desc[i] = 0ull;
             e = 0u;
         }
         ((volatile uint32_t*)p.ctl)[0] = 0u;
@@ -943,6 +945,10 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&fullR[sR]);
             }
+            // start the HBM -> L2 part of the next round's read 1 now
+            const int64_t tn = t + gridDim.x;
+            if (lane == 0 && p.vec && (tn + 1) * (int64_t)TILE <= p.total)
+                prefetch_l2_bulk(in + tn * (int64_t)TILE, TILE * 4);
         }
     } else if (warp == NS + NR + 1) {
         // ---------------- P2: read 2 (from L2) once the carry is known, into ring W
@@ -973,20 +979,26 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         }
     } else {
         // ---------------- NLB look-back warps, tile sequence i handled by warp i mod NLB
+        // speculative: tile ids are static (round robin), so each look-back starts before the
+        // tile's read 1 / reduction; only publishing P waits for this tile's aggregate
+        static_assert(NLB <= SH && SH % NLB == 0, "look-back warps must not lap the header ring");
         const int lb = warp - (NS + NR + 2);
-        for (int64_t i = lb;; i += NLB) {
+        const int64_t n_mine = (num_tiles - blockIdx.x + gridDim.x - 1) / gridDim.x;   // index of the sentinel
+        for (int64_t i = lb; i <= n_mine; i += NLB) {
             const int sH = (int)(i % SH);
-            if (!mbar_wait_or_end(&aggd[sH], (uint32_t)((i / SH) & 1), &s_end, i)) break;
+            const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
+            C carry = Op::cidentity();
+            uint32_t stats[2] = {0u, 0u};
+            if (i < n_mine) {
+                if (lane == 0) trace_stamp(p, t, 4);
+                if (((t * (int64_t)TILE) % p.N) != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            }
+            mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
             SlotHdr<Op, NS>& h = s_hdr[sH];
-            const int64_t t = h.tid;
-            if (t < 0) {
+            if (i == n_mine) {                       // forward the end sentinel to P2
                 if (lane == 0) mbar_arrive(&crd[sH]);
                 break;
             }
-            C carry = Op::cidentity();
-            uint32_t stats[2] = {0u, 0u};
-            if (lane == 0) trace_stamp(p, t, 4);
-            if (h.r != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
             if (lane == 0) {
                 if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
                 h.carry = carry;
@@ -1159,7 +1171,7 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 0: return launch_pipelined<Op, 16, 8, 3, 5, 1, 1>(p, s);  // 64 KiB tiles, window 160, L2 prefetch +1 round
     case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1, 0>(p, s);   // 32 KiB tiles (small, L2-resident totals)
     case 2: return launch_tma<Op, 8, 8>(p, s);                     // one 8192-element tile per CTA
-    case 3: return launch_l2<Op, 8, 4, 3, 3, 32, 10, 4>(p, s);     // two reads (L2-staged), window 320 = 2 rounds
+    case 3: return launch_l2<Op, 8, 4, 3, 3, 8, 5, 8>(p, s);       // two reads (L2-staged), 8-tile header ring, 8 look-back warps
     case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2, 1>(p, s);  // as 0 with two look-back warps
     case 5: return launch_regs<Op, 12, 8, 4, 8, 5, 2>(p, s);       // register-resident waiting tiles, 48 KiB
     case 6: return launch_tma<Op, 8, 4>(p, s);                     // one 4096-element tile per CTA
