@@ -53,10 +53,13 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 //   small totals of few problems (<= 2^22 elements, L2 resident, latency bound): the
 //     paper's three-stage form -- three short kernels beat one persistent look-back launch
 //     in device time (configs[0]: ~6 us vs ~7.5 us).
+//   (boundary re-measured with 64-byte descriptor slots, profiles/r01_boundary.txt: the
+//    look-back matches or beats the CTA cascade up to G = 2048; the cascade wins from
+//    G = 4096, where every SM holds many whole problems)
 scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
-    if (rows_aligned && G >= 592 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
-    if (rows_aligned && G >= 1184 && N >= 1024) return SCAN_ALGO_CASCADE_WARP;
+    if (rows_aligned && G >= 4096 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
+    if (rows_aligned && G >= 1184 && N >= 1024 && N < 4096) return SCAN_ALGO_CASCADE_WARP;
     if (G <= 16 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     return SCAN_ALGO_LOOKBACK;
 }
