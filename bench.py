@@ -301,31 +301,40 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
     x = torch.empty(n_local, dtype=torch.int32, device=dev)
     inputs.fill_device(x, "i32", SEED + 5, offset=rank * n_local)
     y = torch.empty_like(x)
-    comm = multi.NativeComm() if world > 1 else None
+    # the fused exchange (Stage 2 pushes the totals into later ranks' HBM, Stage 3 waits on
+    # the device; no collective call) is the product path; NCCL all-gather beside it
+    comms = {"peer": multi.PeerComm(1) if world > 1 else multi.PeerComm.loopback(1, 1)[0]}
+    if world > 1:
+        comms["nccl"] = multi.NativeComm()
 
-    def run():
+    def run(name):
+        multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
+                         backend="peer" if name == "peer" else "native", comm=comms[name])
+    times = {}
+    for name in comms:
+        for _ in range(3):
+            run(name)
+        torch.cuda.synchronize()
         if world > 1:
-            multi.scan_multi(x, "add", "inclusive", mode="elements", out=y, backend="native", comm=comm)
-        else:
-            t = sb.shard_totals(x, "add")
-            sb.shard_scan(x, t.view(1, -1), 0, 1, "add", "inclusive", out=y)
-    for _ in range(3):
-        run()
+            torch.distributed.barrier()
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record()
+        for _ in range(reps):
+            run(name)
+        s1.record()
+        torch.cuda.synchronize()
+        ms = s0.elapsed_time(s1) / reps
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            ms = float(t.item())
+        times[name] = ms
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
-    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    s0.record()
-    for _ in range(reps):
-        run()
-    s1.record()
-    torch.cuda.synchronize()
-    ms = s0.elapsed_time(s1) / reps
-    if world > 1:
-        t = torch.tensor([ms], device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
-        comm.close()
+    for c in comms.values():
+        c.close()
+    ms = times["peer"]
     # per-phase breakdown (the paper's Fig. 14): Stage 1+2 / exchange /
     # Stage 3, events between the three steps of the torch-backend path
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
@@ -346,7 +355,9 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
     return {"N_total": world * n_local, "N_per_gpu": n_local, "ms": ms,
             "Gelem/s": world * n_local / ms / 1e6, "per_gpu_GB/s_at_12B_per_elem": per_gpu_gbs,
             "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
-            "exchange": "NCCL allgather (scan_batch_multi, native comm)" if world > 1 else "none (W=1)",
+            "exchange": ("fused peer stores in the Stage 2/3 kernels (scan_comm_create_peer)" if world > 1
+                         else "none (W=1; the fused-exchange kernels run with no peers)"),
+            "ms_by_exchange": times,
             "phases_ms_rank%d" % rank: {"stage1+2_reduce": ph[0], "exchange": ph[1], "stage3_scan": ph[2]}}
 
 

@@ -23,7 +23,9 @@ STATUS = {0: "SCAN_OK", 1: "SCAN_ERR_INVALID_ARG", 2: "SCAN_ERR_UNSUPPORTED", 3:
 EXPORTS = ("scan_status_string", "scan_abi_version", "scan_batch", "scan_workspace_bytes",
            "scan_batch_ex", "scan_batch_host", "scan_shard_totals", "scan_shard_scan",
            "scan_shard_workspace_bytes", "scan_debug_trace", "scan_plan", "scan_comm_create_nccl",
-           "scan_comm_get_unique_id", "scan_comm_init_rank", "scan_comm_destroy", "scan_batch_multi")
+           "scan_comm_get_unique_id", "scan_comm_init_rank", "scan_comm_destroy", "scan_batch_multi",
+           "scan_comm_create_peer", "scan_comm_peer_handle", "scan_comm_peer_open")
+PEER_HANDLE_BYTES = 128
 SHARD = {"problems": 0, "elements": 1}
 
 
@@ -56,6 +58,9 @@ def _load() -> ctypes.CDLL:
         "scan_comm_init_rank": ([P, I, I, P], I),
         "scan_comm_destroy": ([P], I),
         "scan_batch_multi": ([P, P, I64, I64, I, I, I, P, I, P, I], I),
+        "scan_comm_create_peer": ([I, I, I64, P], I),
+        "scan_comm_peer_handle": ([P, P], I),
+        "scan_comm_peer_open": ([P, P], I),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)

@@ -191,8 +191,11 @@ ChunkParams chunk_params(const void* in, void* out, int64_t N, int64_t G, scan_k
 scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
                             scan_kind kind, int64_t K, void* ws, const uint64_t* carry_src,
                             int carry_rows, cudaStream_t s, bool stages12, bool stage3,
-                            uint64_t* totals_out) {
+                            uint64_t* totals_out, const PeerParams* peer = nullptr,
+                            int64_t carry_stride = 0) {
     ChunkParams p = chunk_params(in, out, N, G, kind);
+    if (peer) p.peer = *peer;
+    p.carry_stride = carry_stride;
     p.chunk = three_stage_chunk(N, G, K);
     p.Bx = (N + p.chunk - 1) / p.chunk;
     char* base = (char*)ws + kCtlBytes;
@@ -504,3 +507,28 @@ scan_status scan_shard_scan(const void* in_local, void* out_local, int64_t N_loc
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------- fused peer exchange
+// Both halves of one rank's sharded call with the exchange done by the kernels over peer
+// memory (scan_multi.cu owns the mailboxes).  carry rows = ranks < rank of the mailbox.
+scan_status scanb200::shard_run_peer(const void* in, void* out, int64_t N_local, int64_t G, scan_op op,
+                                     scan_dtype dt, scan_kind kind, void* ws, size_t ws_bytes,
+                                     uint64_t* totals, const uint64_t* mailbox_rows, int64_t row_stride,
+                                     const PeerParams& peer, cudaStream_t s) {
+    if (!valid_enums(op, dt, kind)) return SCAN_ERR_INVALID_ARG;
+    int64_t total = 0;
+    scan_status st = check_shape(N_local, G, &total);
+    if (st != SCAN_OK) return st;
+    if (G == 0) return SCAN_OK;
+    if (total > 0) {
+        st = check_buffers(in, out, total, true);
+        if (st != SCAN_OK) return st;
+    }
+    if (ws_bytes < three_stage_bytes(N_local, G, 0)) return SCAN_ERR_NO_MEMORY;
+    st = run_three_stage(in, out, N_local, G, op, dt, kind, 0, ws, mailbox_rows, peer.rank, s, true, false,
+                         totals, &peer, row_stride);
+    if (st != SCAN_OK) return st;
+    if (total == 0) return from_cuda(launch_peer_ack(peer, s));
+    return run_three_stage(in, out, N_local, G, op, dt, kind, 0, ws, mailbox_rows, peer.rank, s, false, true,
+                           totals, &peer, row_stride);
+}

@@ -84,13 +84,28 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     }
 }
 
+// ------------------------------------------------------------------ fused peer exchange
+// Spin helpers of the peer protocol (scan_internal.h, PeerParams).  One thread per CTA
+// spins; the result is published to the CTA by the caller's __syncthreads.
+__device__ __forceinline__ void peer_wait_ge(const uint64_t* slot, uint64_t want) {
+    while (ld_acquire_sys_u64(slot) < want) __nanosleep(64);
+}
+// "Last CTA done" (fence, count, the last one to arrive releases): returns true in
+// exactly one CTA per launch, after every CTA's prior stores are visible system-wide.
+// The counter resets itself for the next launch (stream-ordered after this one).
+__device__ __forceinline__ bool peer_last_cta(uint32_t* counter) {
+    __threadfence_system();
+    const uint32_t n = gridDim.x;
+    if (atomicAdd(counter, 1u) != n - 1) return false;
+    *counter = 0;
+    __threadfence_system();
+    return true;
+}
+
 // ------------------------------------------------------------------ Stage 2
-template <class Op, int WARPS>
-__global__ void __launch_bounds__(WARPS * 32) aux_scan_kernel(ChunkParams p) {
+template <class Op>
+__device__ __forceinline__ void aux_scan_problem(const ChunkParams& p, int64_t g, int lane, bool push) {
     using C = typename Op::Carry;
-    const int warp = threadIdx.x >> 5, lane = lane_id();
-    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
-    if (g >= p.G) return;
     uint64_t* a = p.aux + g * p.Bx;
     C run = Op::cidentity();
     for (int64_t b = 0; b < p.Bx; b += 32) {
@@ -107,7 +122,31 @@ __global__ void __launch_bounds__(WARPS * 32) aux_scan_kernel(ChunkParams p) {
         if (i < p.Bx) a[i] = slot_put(Op::capply(run, ex));
         run = Op::capply(run, shfl_idx_c<C>(incl, 31));
     }
-    if (lane == 0) p.totals[g] = slot_put(run);
+    if (lane == 0) {
+        p.totals[g] = slot_put(run);
+        if (push)       // one-sided stores over NVLink into every later rank's mailbox
+            for (int q = p.peer.rank + 1; q < p.peer.ngpu; ++q) st_relaxed_sys_u64(p.peer.push_totals[q] + g, slot_put(run));
+    }
+}
+
+template <class Op, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) aux_scan_kernel(ChunkParams p) {
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    const PeerParams& pp = p.peer;
+    const bool push = pp.on && pp.rank + 1 < pp.ngpu;      // someone reads this rank's totals
+    if (push) {
+        // the mailbox half this call writes was last read by call epoch-2 of ranks > rank
+        if (threadIdx.x == 0 && pp.epoch > 2)
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) peer_wait_ge(pp.my_acks + q, pp.epoch - 2);
+        __syncthreads();
+    }
+    if (g < p.G) aux_scan_problem<Op>(p, g, lane, push);
+    if (push) {
+        __syncthreads();
+        if (threadIdx.x == 0 && peer_last_cta(pp.counters + 0))
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) st_release_sys_u64(pp.push_flag[q], pp.epoch);
+    }
 }
 
 // ------------------------------------------------------------------ Stage 3 / CTA cascade
@@ -128,7 +167,25 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     // Stage 2 results folded in: carries of earlier ranks (sharded mode),
     // then the exclusive prefix of the chunks before this one.
     C carry = Op::cidentity();
-    for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * p.G + g]));
+    const int64_t stride = p.carry_stride ? p.carry_stride : p.G;
+    if (p.peer.on && p.peer.rank > 0) {
+        // fused exchange: wait for the totals rows of ranks < rank in this rank's mailbox
+        // (pushed by their Stage 2), fold them, and acknowledge once every CTA has read
+        __shared__ C s_carry;
+        if (threadIdx.x == 0) {
+            for (int r = 0; r < p.peer.rank; ++r) peer_wait_ge(p.peer.my_flags + r, p.peer.epoch);
+            C cr = Op::cidentity();
+            for (int r = 0; r < p.carry_rows; ++r)
+                cr = Op::capply(cr, slot_get<C>(ld_relaxed_sys_u64(p.carry_src + (int64_t)r * stride + g)));
+            s_carry = cr;
+            if (peer_last_cta(p.peer.counters + 1))
+                for (int r = 0; r < p.peer.rank; ++r) st_release_sys_u64(p.peer.push_ack[r], p.peer.epoch);
+        }
+        __syncthreads();
+        carry = s_carry;
+    } else {
+        for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
+    }
     if (p.aux) carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
 
     int it = 0;
@@ -164,7 +221,8 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
     const T* in = (const T*)p.in;
     T* out = (T*)p.out;
     C carry = Op::cidentity();
-    for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * p.G + g]));
+    const int64_t stride = p.carry_stride ? p.carry_stride : p.G;
+    for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
     for (int64_t off = 0; off < p.N; off += WCH) {
         WarpTile<Op, false, V> wt;
         wt.load(in, row + off, row + p.N, p.vec);
@@ -172,6 +230,14 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
         wt.store(out, row + off, row + p.N, p.vec, Op::identity(), false, Op::from_carry(carry), p.exclusive);
         carry = Op::capply(carry, Op::to_carry(wt.wtot));
     }
+}
+
+// fused exchange, empty local portion: wait for ranks < rank, acknowledge them
+__global__ void peer_ack_kernel(PeerParams pp) {
+    if (threadIdx.x != 0) return;
+    for (int r = 0; r < pp.rank; ++r) peer_wait_ge(pp.my_flags + r, pp.epoch);
+    __threadfence_system();
+    for (int r = 0; r < pp.rank; ++r) st_release_sys_u64(pp.push_ack[r], pp.epoch);
 }
 
 template <class Op>
@@ -224,5 +290,10 @@ cudaError_t launch_chunk_reduce(OpCode op, const ChunkParams& p, cudaStream_t s)
 cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(auxscan_op) }
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(scan_op) }
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_op) }
+cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s) {
+    if (!pp.on || pp.rank == 0) return cudaSuccess;
+    peer_ack_kernel<<<1, 32, 0, s>>>(pp);
+    return cudaGetLastError();
+}
 
 }  // namespace scanb200

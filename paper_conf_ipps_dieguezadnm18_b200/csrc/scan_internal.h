@@ -4,6 +4,8 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+#include "scan_b200.h"
+
 namespace scanb200 {
 
 enum class OpCode : int { AddU32 = 0, MaxI32 = 1, MaxU32 = 2, MaxF32 = 3, AddF32 = 4 };
@@ -32,6 +34,31 @@ int64_t lookback_tile_elems(int variant);
 int lookback_num_variants();
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s);
 
+// ---------------------------------------------------------------- fused peer exchange
+// The exchange step of the sharded path done by the kernels themselves over peer memory
+// (Stage 1 results of every GPU reach the GPUs that need them; here by
+// one-sided NVLink stores instead of P2P copies to a master GPU).  Every rank owns a
+// mailbox in its own HBM (layout in scan_multi.cu); peers write into it, it only reads it.
+//   Stage 2 (aux_scan)  waits until every rank p > rank acknowledged call epoch-2 (the
+//                       mailbox parity it is about to overwrite), stores its G portion
+//                       totals into row `rank` of every peer p > rank, and the last CTA
+//                       release-stores `epoch` into flag[rank] of those peers.
+//   Stage 3 (chunk_scan) acquire-spins on its own flags of ranks < rank, folds their rows
+//                       into the carry, and the last CTA release-stores `epoch` into
+//                       ack[rank] of every peer p < rank.
+constexpr int kMaxPeers = 8;
+struct PeerParams {
+    uint64_t* push_totals[kMaxPeers];   // peer p's mailbox row `rank` of this call's parity
+    uint64_t* push_flag[kMaxPeers];     // &flags[rank] in peer p's mailbox
+    uint64_t* push_ack[kMaxPeers];      // &acks[rank] in peer p's mailbox
+    const uint64_t* my_flags;           // own mailbox flags[kMaxPeers] (written by ranks < rank)
+    const uint64_t* my_acks;            // own mailbox acks[kMaxPeers]  (written by ranks > rank)
+    uint32_t* counters;                 // own mailbox: [0] Stage 2, [1] Stage 3 CTAs done
+    uint64_t epoch;                     // this call's number (>= 1), identical on every rank
+    int rank, ngpu;
+    bool on;
+};
+
 // ---------------------------------------------------------------- cascade / three-stage
 // Chunked per-problem kernels.  Problem g is cut into Bx chunks of `chunk` elements
 // (chunk = K * tile, the paper's cascade depth K).
@@ -46,8 +73,10 @@ struct ChunkParams {
     uint64_t* totals;       // [G] problem totals (Stage 2 output)
     const uint64_t* carry_src;  // [carry_rows][G] slots folded into every problem's carry
     int carry_rows;
+    int64_t carry_stride;   // elements between carry rows (0 means G)
     bool vec;
     bool exclusive;
+    PeerParams peer;        // fused exchange (peer.on) -- sharded path only
 };
 int64_t chunk_tile_elems();
 int64_t warp_tile_elems();
@@ -61,5 +90,16 @@ cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 // Warp-per-problem cascade (L_y = warps per block problems per CTA).
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Fused exchange with an empty local portion (no Stage 3 CTAs): one CTA waits for the
+// flags of ranks < rank and acknowledges them, so peers never wait on this rank.
+cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s);
+
+// Host side of the fused exchange (scan_api.cu): Stage 1+2 with the push, Stage 3 with
+// the wait and the acknowledgement, on one stream.  `ws` must be sized by
+// three_stage_bytes(N_local, G, 0) (scan_shard_workspace_bytes).
+scan_status shard_run_peer(const void* in, void* out, int64_t N_local, int64_t G, scan_op op, scan_dtype dt,
+                           scan_kind kind, void* ws, size_t ws_bytes, uint64_t* totals,
+                           const uint64_t* mailbox_rows, int64_t row_stride, const PeerParams& peer,
+                           cudaStream_t s);
 
 }  // namespace scanb200

@@ -16,9 +16,12 @@ Two ways to use several GPUs (PAPER.md:191-193 [§4]):
 
 ``backend="torch"`` does the exchange with ``torch.distributed.all_gather_into_tensor``
 on the caller's process group; ``backend="native"`` calls the C-ABI
-``scan_batch_multi`` with the group's own NCCL communicator (one library call per rank).
-All device work runs in libscanb200.so; only the sharding plan and the collective call
-are Python.
+``scan_batch_multi`` with the group's own NCCL communicator (one library call per rank);
+``backend="peer"`` (:class:`PeerComm`) makes no collective call at all: the Stage 2
+kernel stores the totals straight into the later ranks' HBM over NVLink and the Stage 3
+kernel waits for them on the device (the paper's P2P writes, fused
+into the kernels).  All device work runs in libscanb200.so; only the sharding plan, the
+one-time handle exchange and the collective call are Python.
 """
 from __future__ import annotations
 
@@ -30,7 +33,8 @@ import torch.distributed as dist
 from . import _lib, shard_scan, shard_totals
 from ._lib import KINDS, OPS, check
 
-__all__ = ["partition", "grouped_plan", "make_groups", "exchange_totals", "scan_multi", "NativeComm"]
+__all__ = ["partition", "grouped_plan", "make_groups", "exchange_totals", "scan_multi", "NativeComm",
+           "PeerComm"]
 
 
 def partition(n: int, world: int, rank: int) -> tuple[int, int]:
@@ -104,9 +108,57 @@ class NativeComm:
             self.handle = None
 
 
+class PeerComm:
+    """scan_comm_t with the fused exchange over peer memory (scan_comm_create_peer).
+
+    Setup (collective over ``group``, any backend -- gloo works): every rank creates its
+    mailbox for ``max_G`` problems, the handles are all-gathered once, every rank maps the
+    others'.  Afterwards ``scan_multi(..., backend="peer", comm=self)`` runs with no
+    collective call.  ``PeerComm.loopback(W, max_G)`` builds W communicators inside one
+    process (virtual ranks on one device, for tests)."""
+
+    def __init__(self, max_G: int, group=None, *, rank: int | None = None, world: int | None = None,
+                 _open: bool = True):
+        self.rank = dist.get_rank(group) if rank is None else rank
+        self.world = dist.get_world_size(group) if world is None else world
+        h = ctypes.c_void_p(0)
+        check("scan_comm_create_peer", _lib.lib.scan_comm_create_peer(self.rank, self.world, int(max_G),
+                                                                        ctypes.byref(h)))
+        self.handle = h
+        self.max_G = int(max_G)
+        if _open:
+            blobs = [None] * self.world
+            dist.all_gather_object(blobs, self.peer_handle(), group=group)
+            self.open(blobs)
+
+    def peer_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(_lib.PEER_HANDLE_BYTES)
+        check("scan_comm_peer_handle", _lib.lib.scan_comm_peer_handle(self.handle, buf))
+        return buf.raw
+
+    def open(self, blobs) -> None:
+        if len(blobs) != self.world or any(len(b) != _lib.PEER_HANDLE_BYTES for b in blobs):
+            raise ValueError("need one %d-byte handle per rank" % _lib.PEER_HANDLE_BYTES)
+        allb = ctypes.create_string_buffer(b"".join(blobs), len(blobs) * _lib.PEER_HANDLE_BYTES)
+        check("scan_comm_peer_open", _lib.lib.scan_comm_peer_open(self.handle, allb))
+
+    @classmethod
+    def loopback(cls, world: int, max_G: int) -> list["PeerComm"]:
+        comms = [cls(max_G, rank=r, world=world, _open=False) for r in range(world)]
+        blobs = [c.peer_handle() for c in comms]
+        for c in comms:
+            c.open(blobs)
+        return comms
+
+    def close(self):
+        if self.handle:
+            check("scan_comm_destroy", _lib.lib.scan_comm_destroy(self.handle))
+            self.handle = None
+
+
 def scan_multi(x_local: torch.Tensor, op: str = "add", kind: str = "inclusive", mode: str = "elements",
                group=None, out: torch.Tensor | None = None, backend: str = "torch",
-               comm: NativeComm | None = None) -> torch.Tensor:
+               comm: "NativeComm | PeerComm | None" = None) -> torch.Tensor:
     """Scan this rank's share.  ``x_local`` is (G, N_local) or (N_local,).
 
     mode="problems": x_local holds whole problems (this rank's partition of the batch).
@@ -123,9 +175,12 @@ def scan_multi(x_local: torch.Tensor, op: str = "add", kind: str = "inclusive", 
         return scan_local(x_local, op, kind, out=out)
     if mode != "elements":
         raise ValueError(mode)
-    if backend == "native":
-        c = comm if comm is not None else NativeComm(group)
+    if backend in ("native", "peer"):
         N, G = (x_local.shape[0], 1) if x_local.dim() == 1 else (x_local.shape[1], x_local.shape[0])
+        if comm is not None:
+            c = comm
+        else:
+            c = NativeComm(group) if backend == "native" else PeerComm(G, group)
         from . import _dtype, _stream
         rc = _lib.lib.scan_batch_multi(x_local.data_ptr(), out.data_ptr(), N, G, OPS[op], _dtype(x_local),
                                        KINDS[kind], _stream(x_local, None), c.world, c.handle,
@@ -133,6 +188,8 @@ def scan_multi(x_local: torch.Tensor, op: str = "add", kind: str = "inclusive", 
         check("scan_batch_multi", rc)
         if comm is None:
             torch.cuda.current_stream().synchronize()
+            if backend == "peer":         # peers may still write acks into this mailbox
+                dist.barrier(group)
             c.close()
         return out
     totals = shard_totals(x_local, op)                        # Stage 1 + 2 (local)
