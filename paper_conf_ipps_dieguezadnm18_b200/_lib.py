@@ -73,7 +73,7 @@ lib = _load()
 
 
 def lib_num_lookback_variants() -> int:
-    return 10
+    return 13
 
 
 def check(fn: str, code: int) -> None:

@@ -72,6 +72,9 @@ int choose_lookback_variant(int64_t N, int64_t G) {
 int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
     const int64_t tile = chunk_tile_elems();
     if (K > 0) return K * tile;
+    // latency-bound totals (configs[0]): two tiles per chunk measured best on B200
+    // (2^20: 5.1 us at K = 2 against 5.9 us at K = 1 and 6.6 us at K = 3, CUDA graph)
+    if (N * G <= (int64_t(1) << 22)) return 2 * tile;
     int64_t bx = std::max<int64_t>(1, (kTargetCtas + G - 1) / G);
     int64_t chunk = (N + bx - 1) / bx;
     chunk = std::max<int64_t>(tile, (chunk + tile - 1) / tile * tile);
@@ -192,7 +195,7 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
                             scan_kind kind, int64_t K, void* ws, const uint64_t* carry_src,
                             int carry_rows, cudaStream_t s, bool stages12, bool stage3,
                             uint64_t* totals_out, const PeerParams* peer = nullptr,
-                            int64_t carry_stride = 0) {
+                            int64_t carry_stride = 0, bool pdl3 = false) {
     ChunkParams p = chunk_params(in, out, N, G, kind);
     if (peer) p.peer = *peer;
     p.carry_stride = carry_stride;
@@ -205,11 +208,15 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
     p.carry_rows = carry_rows;
     const OpCode oc = opcode(op, dt);
     if (stages12) {
-        cudaError_t e = launch_chunk_reduce(oc, p, s);
+        cudaError_t e = launch_chunk_reduce(oc, p, s);       // normal launch: waits for the caller's work
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
+        p.pdl = true;                                        // Stage 2 overlaps Stage 1's tail
         e = launch_aux_scan(oc, p, s);
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
     }
+    // Stage 3 directly after this library's Stage 2 (same call, or the fused-exchange
+    // path) starts early and loads its first tile while Stage 2 finishes
+    p.pdl = stages12 || pdl3;
     if (stage3) return from_cuda(launch_chunk_scan(oc, p, s));
     return SCAN_OK;
 }
@@ -530,5 +537,5 @@ scan_status scanb200::shard_run_peer(const void* in, void* out, int64_t N_local,
     if (st != SCAN_OK) return st;
     if (total == 0) return from_cuda(launch_peer_ack(peer, s));
     return run_three_stage(in, out, N_local, G, op, dt, kind, 0, ws, mailbox_rows, peer.rank, s, false, true,
-                           totals, &peer, row_stride);
+                           totals, &peer, row_stride, true);
 }

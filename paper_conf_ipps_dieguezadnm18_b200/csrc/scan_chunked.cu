@@ -60,6 +60,7 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     const int64_t start = c * p.chunk;
     const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
     const T* in = (const T*)p.in;
+    grid_dep_launch();          // Stage 2 may be scheduled now; it waits for our results
 
     C acc = Op::cidentity();
     for (int64_t off = start + warp * WCH; off < end; off += TILE) {
@@ -135,6 +136,8 @@ __global__ void __launch_bounds__(WARPS * 32) aux_scan_kernel(ChunkParams p) {
     const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
     const PeerParams& pp = p.peer;
     const bool push = pp.on && pp.rank + 1 < pp.ngpu;      // someone reads this rank's totals
+    grid_dep_launch();          // Stage 3 may be scheduled now (it loads its data meanwhile)
+    grid_dep_wait();            // Stage 1's chunk reductions are complete and visible
     if (push) {
         // the mailbox half this call writes was last read by call epoch-2 of ranks > rank
         if (threadIdx.x == 0 && pp.epoch > 2)
@@ -165,34 +168,40 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     T* out = (T*)p.out;
 
     // Stage 2 results folded in: carries of earlier ranks (sharded mode),
-    // then the exclusive prefix of the chunks before this one.
-    C carry = Op::cidentity();
-    const int64_t stride = p.carry_stride ? p.carry_stride : p.G;
-    if (p.peer.on && p.peer.rank > 0) {
-        // fused exchange: wait for the totals rows of ranks < rank in this rank's mailbox
-        // (pushed by their Stage 2), fold them, and acknowledge once every CTA has read
-        __shared__ C s_carry;
-        if (threadIdx.x == 0) {
-            for (int r = 0; r < p.peer.rank; ++r) peer_wait_ge(p.peer.my_flags + r, p.peer.epoch);
-            C cr = Op::cidentity();
-            for (int r = 0; r < p.carry_rows; ++r)
-                cr = Op::capply(cr, slot_get<C>(ld_relaxed_sys_u64(p.carry_src + (int64_t)r * stride + g)));
-            s_carry = cr;
-            if (peer_last_cta(p.peer.counters + 1))
-                for (int r = 0; r < p.peer.rank; ++r) st_release_sys_u64(p.peer.push_ack[r], p.peer.epoch);
+    // then the exclusive prefix of the chunks before this one.  Read after
+    // the first tile's loads are in flight: launched as a dependent of Stage 2 (p.pdl), the
+    // CTA starts while Stage 2 still runs and only grid_dep_wait() orders the reads below.
+    auto fold_carry = [&]() -> C {
+        grid_dep_wait();
+        C carry = Op::cidentity();
+        const int64_t stride = p.carry_stride ? p.carry_stride : p.G;
+        if (p.peer.on && p.peer.rank > 0) {
+            // fused exchange: wait for the totals rows of ranks < rank in this rank's mailbox
+            // (pushed by their Stage 2), fold them, and acknowledge once every CTA has read
+            __shared__ C s_carry;
+            if (threadIdx.x == 0) {
+                for (int r = 0; r < p.peer.rank; ++r) peer_wait_ge(p.peer.my_flags + r, p.peer.epoch);
+                C cr = Op::cidentity();
+                for (int r = 0; r < p.carry_rows; ++r)
+                    cr = Op::capply(cr, slot_get<C>(ld_relaxed_sys_u64(p.carry_src + (int64_t)r * stride + g)));
+                s_carry = cr;
+                if (peer_last_cta(p.peer.counters + 1))
+                    for (int r = 0; r < p.peer.rank; ++r) st_release_sys_u64(p.peer.push_ack[r], p.peer.epoch);
+            }
+            __syncthreads();
+            carry = s_carry;
+        } else {
+            for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
         }
-        __syncthreads();
-        carry = s_carry;
-    } else {
-        for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
-    }
-    if (p.aux) carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
+        if (p.aux) carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
+        return carry;
+    };
+    C carry = Op::cidentity();
 
-    int it = 0;
-    for (int64_t off = start; off < end; off += TILE, ++it) {
-        WarpTile<Op, false, V> wt;
+    // one tile: scan, block combine, store with the running carry (the cascade, Fig. 5)
+    auto process = [&](WarpTile<Op, false, V>& wt, int64_t off, int it) {
         const int64_t wb = row + off + warp * WCH;
-        wt.load(in, wb, row + end, p.vec);
+        if (it == 0) carry = fold_carry();
         wt.scan();
         if (lane == 0) s_wval[it & 1][warp] = wt.wtot;
         __syncthreads();
@@ -204,7 +213,23 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
             tot = Op::apply(tot, v);
         }
         wt.store(out, wb, row + end, p.vec, wp, false, Op::from_carry(carry), p.exclusive);
-        carry = Op::capply(carry, Op::to_carry(tot));       // the cascade carry (Fig. 5)
+        carry = Op::capply(carry, Op::to_carry(tot));
+    };
+    // software pipeline over the chunk's tiles: the loads of tile i+1 are issued before
+    // tile i is scanned, so every thread keeps two tiles' rows in flight (ping-pong
+    // registers A/B, compile-time indexed)
+    WarpTile<Op, false, V> A, B;
+    int it = 0;
+    int64_t off = start;
+    if (off < end) A.load(in, row + off + warp * WCH, row + end, p.vec);
+    while (off < end) {
+        if (off + TILE < end) B.load(in, row + off + TILE + warp * WCH, row + end, p.vec);
+        process(A, off, it++);
+        off += TILE;
+        if (off >= end) break;
+        if (off + TILE < end) A.load(in, row + off + TILE + warp * WCH, row + end, p.vec);
+        process(B, off, it++);
+        off += TILE;
     }
 }
 
@@ -248,20 +273,37 @@ cudaError_t reduce_op(const ChunkParams& p, cudaStream_t s) {
     chunk_reduce_kernel<Op, CH_WARPS, CH_V><<<(unsigned)blocks, CH_WARPS * 32, 0, s>>>(p);
     return cudaGetLastError();
 }
+// launch, as a programmatic dependent of the stream's previous kernel when p.pdl
+template <class Kern>
+cudaError_t launch_maybe_pdl(Kern kern, unsigned blocks, unsigned threads, const ChunkParams& p, cudaStream_t s) {
+    if (!p.pdl) {
+        kern<<<blocks, threads, 0, s>>>(p);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(blocks);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, p);
+}
 template <class Op>
 cudaError_t auxscan_op(const ChunkParams& p, cudaStream_t s) {
     int64_t blocks = (p.G + 7) / 8;
     if (blocks == 0) return cudaSuccess;
-    aux_scan_kernel<Op, 8><<<(unsigned)blocks, 8 * 32, 0, s>>>(p);
-    return cudaGetLastError();
+    return launch_maybe_pdl(aux_scan_kernel<Op, 8>, (unsigned)blocks, 8 * 32, p, s);
 }
 template <class Op>
 cudaError_t scan_op(const ChunkParams& p, cudaStream_t s) {
     int64_t blocks = p.G * p.Bx;
     if (blocks == 0) return cudaSuccess;
     if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    chunk_scan_kernel<Op, CH_WARPS, CH_V><<<(unsigned)blocks, CH_WARPS * 32, 0, s>>>(p);
-    return cudaGetLastError();
+    return launch_maybe_pdl(chunk_scan_kernel<Op, CH_WARPS, CH_V>, (unsigned)blocks, CH_WARPS * 32, p, s);
 }
 template <class Op>
 cudaError_t warp_op(const ChunkParams& p, cudaStream_t s) {

@@ -152,6 +152,13 @@ __device__ __forceinline__ void st_relaxed_f64(double* p, double v) {
     asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" :: "l"(p), "d"(v) : "memory");
 }
 
+// Programmatic dependent launch (sm_90+): a kernel launched with the
+// programmatic-stream-serialization attribute may start while the previous kernel of the
+// stream still runs; `grid_dep_wait` blocks until that kernel completed and its memory is
+// visible (a no-op for a normal launch); `grid_dep_launch` lets the next kernel start.
+__device__ __forceinline__ void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void grid_dep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // system scope: the fused peer-memory exchange of the sharded path (other GPUs' memory
 // mapped into this address space over NVLink, or another process's memory on this GPU)
 __device__ __forceinline__ void st_release_sys_u64(uint64_t* p, uint64_t v) {

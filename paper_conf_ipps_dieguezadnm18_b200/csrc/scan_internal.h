@@ -76,6 +76,8 @@ struct ChunkParams {
     int64_t carry_stride;   // elements between carry rows (0 means G)
     bool vec;
     bool exclusive;
+    bool pdl;               // launch as a programmatic dependent of the previous kernel of
+                            // this library call (Stage 2 after Stage 1, Stage 3 after Stage 2)
     PeerParams peer;        // fused exchange (peer.on) -- sharded path only
 };
 int64_t chunk_tile_elems();

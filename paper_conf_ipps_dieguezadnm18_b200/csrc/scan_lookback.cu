@@ -1089,6 +1089,82 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
     if (threadIdx.x == 0) epilogue(p);
 }
 
+// ---------------------------------------------------------------- one register tile per CTA
+// Latency-bound totals (configs[0]: 2^20 elements = 128 tiles, L2-resident).  Every thread
+// holds its V 128-bit rows in registers (no shared-memory staging, one pass); the CTA's
+// aggregate is published as soon as the block combine is done and the last warp looks
+// back while the others wait at one barrier; then everyone adds the carry and stores.
+// Tiles follow blockIdx (in-order dispatch, as lookback_tma_kernel).
+template <class Op, bool SEG, int WARPS, int V>
+__device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t tile, uint32_t tag, int64_t r,
+                                             typename Op::T* s_wval, uint32_t* s_wflag, typename Op::Carry* s_carry) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t wb = tile * (int64_t)TILE + warp * WCH;
+    const T* in = (const T*)p.in;
+    WarpTile<Op, SEG, V> wt;
+    if (threadIdx.x == 0) trace_stamp(p, tile, 7);
+    wt.load(in, wb, p.total, p.vec);
+    if (SEG) {
+        const bool small = p.N < TILE;
+        const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+        wt.heads(warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+    }
+    wt.scan();
+    if (lane == 0) { s_wval[warp] = wt.wtot; s_wflag[warp] = wt.wfl; }
+    __syncthreads();
+    T wp = Op::identity(); bool wpf = false;
+#pragma unroll
+    for (int w = 0; w < WARPS; ++w) {
+        if (w < warp) {
+            T v = s_wval[w]; bool f = SEG && s_wflag[w];
+            wp = SEG ? seg_fold<Op>(wp, f, v) : Op::apply(wp, v);
+            wpf = wpf || f;
+        }
+    }
+    if (warp == WARPS - 1) {
+        T agg = SEG ? seg_fold<Op>(wp, wt.wfl, wt.wtot) : Op::apply(wp, wt.wtot);
+        const bool starts = (r == 0);
+        const bool has_head = SEG ? (wpf || wt.wfl) : starts;
+        const C aggc = Op::to_carry(agg);
+        if (lane == 0) { trace_stamp(p, tile, 0); Desc<Op>::publish(p, tile, tag, has_head ? ST_P : ST_A, aggc); }
+        if (lane == 0) { trace_stamp(p, tile, 1); trace_stamp(p, tile, 4); }
+        C carry = Op::cidentity();
+        uint32_t stats[2] = {0u, 0u};
+        if (!starts) carry = look_back<Op>(p, tile, tag, p.trace ? stats : nullptr);
+        if (lane == 0) {
+            if (!has_head) Desc<Op>::publish(p, tile, tag, ST_P, Op::capply(carry, aggc));
+            trace_stamp(p, tile, 2);
+            trace_value(p, tile, 5, stats[0]);
+            trace_value(p, tile, 6, stats[1]);
+            *s_carry = carry;
+        }
+    }
+    __syncthreads();
+    wt.store((T*)p.out, wb, p.total, p.vec, wp, wpf, Op::from_carry(*s_carry), p.exclusive);
+    if (threadIdx.x == 0) trace_stamp(p, tile, 3);
+}
+
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4;
+    __shared__ T s_wval[WARPS];
+    __shared__ uint32_t s_wflag[WARPS];
+    __shared__ C s_carry;
+    const int64_t tile = blockIdx.x;
+    const TileInfo ti = classify(p, tile, TILE);
+    const uint32_t tag = read_tag(p);
+    if (ti.seg) regtile_body<Op, true, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
+    else        regtile_body<Op, false, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
 // ---------------------------------------------------------------- launchers
 int g_num_sms = 0;
 
@@ -1141,6 +1217,15 @@ cudaError_t launch_tma(const LookbackParams& p, cudaStream_t s) {
     return cudaGetLastError();
 }
 
+template <class Op, int WARPS, int V>
+cudaError_t launch_regtile(const LookbackParams& p, cudaStream_t s) {
+    constexpr int TILE = WARPS * 32 * V * 4;
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    lookback_regtile_kernel<Op, WARPS, V><<<(unsigned)tiles, WARPS * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
 template <class Op, int WARPS, int V, int S, int M, int NLB, int PF = 0>
 cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
@@ -1177,6 +1262,9 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 6: return launch_tma<Op, 8, 4>(p, s);                     // one 4096-element tile per CTA
     case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);      // 16 KiB tiles, 4-slot ring
     case 8: return launch_pipelined<Op, 18, 8, 3, 5, 1, 2>(p, s);  // 72 KiB tiles, L2 prefetch +2 rounds
+    case 10: return launch_regtile<Op, 16, 4>(p, s);               // one 8192-element register tile per CTA
+    case 11: return launch_regtile<Op, 8, 4>(p, s);                // one 4096-element register tile per CTA
+    case 12: return launch_regtile<Op, 32, 4>(p, s);               // one 16384-element register tile per CTA
     default: return launch_pipelined<Op, 16, 8, 3, 5, 1, 0>(p, s); // as 0 without the L2 prefetch
     }
 }
@@ -1184,10 +1272,10 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
 }  // namespace
 
 int64_t lookback_tile_elems(int variant) {
-    return (variant == 0 || variant == 4 || variant == 9) ? 16384 : variant == 5 ? 12288
-         : variant == 8 ? 18432 : (variant == 6 || variant == 7) ? 4096 : 8192;
+    return (variant == 0 || variant == 4 || variant == 9 || variant == 12) ? 16384 : variant == 5 ? 12288
+         : variant == 8 ? 18432 : (variant == 6 || variant == 7 || variant == 11) ? 4096 : 8192;
 }
-int lookback_num_variants() { return 10; }
+int lookback_num_variants() { return 13; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

@@ -92,7 +92,7 @@ def test_binding_fails_loudly_without_library(tmp_path, monkeypatch):
 
 
 def test_lookback_variant_count_matches_library():
-    # tests/test_gpu_parity.py::test_lookback_variants covers range(10); the binding and
+    # tests/test_gpu_parity.py::test_lookback_variants covers range(13); the binding and
     # the library must agree on how many variants exist
     from paper_conf_ipps_dieguezadnm18_b200 import _lib
-    assert _lib.lib_num_lookback_variants() == 10
+    assert _lib.lib_num_lookback_variants() == 13

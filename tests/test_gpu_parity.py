@@ -39,7 +39,7 @@ def test_shapes_all_algos(algo, op, dt, kind):
             assert_parity(got, x, op, kind, label="%s %s %s %s N=%d G=%d" % (algo, op, dt, kind, N, G))
 
 
-@pytest.mark.parametrize("variant", range(10))
+@pytest.mark.parametrize("variant", range(13))
 def test_lookback_variants(variant):
     for op, dt in COMBOS:
         for N, G in [(1, 3000), (3, 5000), (100, 333), (8193, 5), (65536 + 17, 3), (1 << 20, 1)]:

@@ -25,7 +25,8 @@ x = torch.empty(a.G * a.N, dtype=torch.int32, device="cuda")
 inputs.fill_device(x, {"i32": "i32", "f32": "f32u"}[a.dtype], 7)
 x = x.view(dt).view(a.G, a.N)
 y = torch.empty_like(x)
-TILE = a.tile or {0: 16384, 4: 16384, 9: 16384, 5: 12288, 8: 18432, 6: 4096, 7: 4096}.get(a.param, 8192)
+TILE = a.tile or {0: 16384, 4: 16384, 9: 16384, 5: 12288, 8: 18432, 6: 4096, 7: 4096, 11: 4096,
+                  12: 16384}.get(a.param, 8192)
 tiles = (a.G * a.N + TILE - 1) // TILE
 tr = torch.zeros(tiles * 8, dtype=torch.int64, device="cuda")
 for _ in range(3):
@@ -46,6 +47,11 @@ def pct(v, name, scale=1e3, unit="us"):
         name, *np.percentile(v, [10, 50, 90, 99]), v.mean(), unit))
 
 
+if R[:, 7].any():          # register-tile kernels also stamp the CTA entry (slot 7)
+    E = R[:, 7] - R[:, 7].min()
+    Z = R[:, :5] - R[:, 7].min()
+    print("entry spread us %.2f; first entry -> last written us %.2f" % (E.max() / 1e3, Z[:, 3].max() / 1e3))
+    pct(R[:, 0] - R[:, 7], "entry -> ready (load+scan)")
 pct(T[:, 1] - T[:, 0], "ready -> A (pass1)")
 pct(T[:, 4] - T[:, 1], "A -> look-back start (queue)")
 pct(T[:, 2] - T[:, 4], "look-back duration")
