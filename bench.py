@@ -291,11 +291,12 @@ def extras(sb, dev):
     return out
 
 
-def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
-    """configs[4]-style sharded single problem (Multi-GPU Problem Scattering):
-    each rank owns a contiguous 2^28-element int32 portion of ONE problem; Stage 1+2 ->
-    NCCL all-gather of the rank totals -> Stage 3.  Weak-scaled (N = W x 2^28).  At W = 1 the
-    same two-pass pipeline runs without the collective (its 1-GPU reference rate)."""
+def elements_mode(sb, dev, world, rank, n_local=1 << 33, reps=10):
+    """configs[4]: one int32 add-scan sharded by elements (Multi-GPU Problem Scattering,
+    PAPER.md:195-205): each rank owns a contiguous 2^33-element portion (32 GiB in + 32 GiB
+    out) of ONE problem -- at W = 8 the problem is configs[4]'s N = 2^36.  Stage 1+2 ->
+    exchange -> Stage 3.  Weak-scaled (N = W x 2^33).  At W = 1 the same two-pass pipeline
+    runs with no peer (its 1-GPU reference rate)."""
     import inputs
     from paper_conf_ipps_dieguezadnm18_b200 import multi
     x = torch.empty(n_local, dtype=torch.int32, device=dev)
@@ -339,9 +340,11 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 28, reps=10):
     # Stage 3, events between the three steps of the torch-backend path
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
     ph = [0.0, 0.0, 0.0]
+    t = sb.shard_totals(x, "add")                 # warm-up (workspace growth), totals reused
+    torch.cuda.synchronize()
     for _ in range(reps):
         ev[0].record()
-        t = sb.shard_totals(x, "add")
+        sb.shard_totals(x, "add", totals=t)
         ev[1].record()
         allt = multi.exchange_totals(t) if world > 1 else t.view(1, -1)
         ev[2].record()
@@ -516,6 +519,7 @@ def main():
     if not args.no_extras:
         el = elements_mode(sb, dev, world, rank)
         res["elements_mode_sharded_problem"] = el
+        torch.cuda.empty_cache()
     if rank == 0 and not args.no_e2e:
         res["e2e"] = e2e(sb)
     if rank == 0 and world == 1 and not args.no_cpu:

@@ -88,8 +88,23 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
 // ------------------------------------------------------------------ fused peer exchange
 // Spin helpers of the peer protocol (scan_internal.h, PeerParams).  One thread per CTA
 // spins; the result is published to the CTA by the caller's __syncthreads.
+// A peer that never arrives (a rank that crashed, or calls issued out of order) must not
+// hang the device forever: after kPeerTimeoutNs the kernel traps, which surfaces as a CUDA
+// error at the caller's next synchronisation ("fail loudly").
+constexpr uint64_t kPeerTimeoutNs = 120ull * 1000000000ull;
+__device__ __forceinline__ uint64_t global_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 __device__ __forceinline__ void peer_wait_ge(const uint64_t* slot, uint64_t want) {
-    while (ld_acquire_sys_u64(slot) < want) __nanosleep(64);
+    if (ld_acquire_sys_u64(slot) >= want) return;
+    const uint64_t t0 = global_ns();
+    uint32_t n = 0;
+    while (ld_acquire_sys_u64(slot) < want) {
+        __nanosleep(64);
+        if ((++n & 1023u) == 0u && global_ns() - t0 > kPeerTimeoutNs) __trap();
+    }
 }
 // "Last CTA done" (fence, count, the last one to arrive releases): returns true in
 // exactly one CTA per launch, after every CTA's prior stores are visible system-wide.
@@ -127,6 +142,60 @@ __device__ __forceinline__ void aux_scan_problem(const ChunkParams& p, int64_t g
         p.totals[g] = slot_put(run);
         if (push)       // one-sided stores over NVLink into every later rank's mailbox
             for (int q = p.peer.rank + 1; q < p.peer.ngpu; ++q) st_relaxed_sys_u64(p.peer.push_totals[q] + g, slot_put(run));
+    }
+}
+
+// One CTA per problem, for many chunks per problem (large portions cut into short chunks
+// so that concurrently running Stage 1/3 CTAs touch neighbouring memory): the Bx chunk
+// values are scanned 32*WARPS at a time (warp shuffles + one smem slot per warp, the same
+// block combine as the tile kernels).
+template <class Op, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) aux_scan_cta_kernel(ChunkParams p) {
+    using C = typename Op::Carry;
+    __shared__ C s_w[WARPS];
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = blockIdx.x;
+    const PeerParams& pp = p.peer;
+    const bool push = pp.on && pp.rank + 1 < pp.ngpu;
+    grid_dep_launch();
+    grid_dep_wait();
+    if (push) {
+        if (threadIdx.x == 0 && pp.epoch > 2)
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) peer_wait_ge(pp.my_acks + q, pp.epoch - 2);
+        __syncthreads();
+    }
+    uint64_t* a = p.aux + g * p.Bx;
+    C run = Op::cidentity();
+    for (int64_t b = 0; b < p.Bx; b += WARPS * 32) {
+        const int64_t i = b + threadIdx.x;
+        const C v = i < p.Bx ? slot_get<C>(a[i]) : Op::cidentity();
+        C incl = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            C y = shfl_up_c<C>(incl, d);
+            if (lane >= d) incl = Op::capply(y, incl);
+        }
+        if (lane == 31) s_w[warp] = incl;
+        __syncthreads();
+        C wp = Op::cidentity(), btot = Op::cidentity();
+#pragma unroll 4
+        for (int w = 0; w < WARPS; ++w) {
+            const C t = s_w[w];
+            if (w < warp) wp = Op::capply(wp, t);
+            btot = Op::capply(btot, t);
+        }
+        C ex = shfl_up_c<C>(incl, 1);
+        if (lane == 0) ex = Op::cidentity();
+        if (i < p.Bx) a[i] = slot_put(Op::capply(Op::capply(run, wp), ex));
+        run = Op::capply(run, btot);
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        p.totals[g] = slot_put(run);
+        if (push)
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) st_relaxed_sys_u64(pp.push_totals[q] + g, slot_put(run));
+        if (push && peer_last_cta(pp.counters + 0))
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) st_release_sys_u64(pp.push_flag[q], pp.epoch);
     }
 }
 
@@ -294,6 +363,10 @@ cudaError_t launch_maybe_pdl(Kern kern, unsigned blocks, unsigned threads, const
 }
 template <class Op>
 cudaError_t auxscan_op(const ChunkParams& p, cudaStream_t s) {
+    if (p.Bx > 256) {               // many chunks per problem: a CTA per problem
+        if (p.G > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+        return launch_maybe_pdl(aux_scan_cta_kernel<Op, 32>, (unsigned)p.G, 32 * 32, p, s);
+    }
     int64_t blocks = (p.G + 7) / 8;
     if (blocks == 0) return cudaSuccess;
     return launch_maybe_pdl(aux_scan_kernel<Op, 8>, (unsigned)blocks, 8 * 32, p, s);

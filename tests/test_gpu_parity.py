@@ -59,6 +59,20 @@ def test_three_stage_cascade_depth(K):
     assert_parity(got, x, "add", "inclusive")
 
 
+def test_three_stage_many_chunks():
+    # long portions are cut into <= 16-tile chunks; more than 256 chunks per problem switch
+    # Stage 2 to one CTA per problem (1024 chunk values per round, ragged last round)
+    for op, dt in COMBOS:
+        for G, N in [(1, (1 << 25) + 12345), (2, 300 * 65536 + 7)]:
+            x = inputs.generate(DIST[dt], G * N, seed=N % 977).reshape(G, N)
+            for kind in ("inclusive", "exclusive"):
+                got = _run(x, op, kind, "three_stage", 0)
+                assert_parity(got, x, op, kind, label="3stage-many %s %s %s G=%d" % (op, dt, kind, G))
+            if op == "add" and dt == "i32":
+                got1 = _run(x, op, "inclusive", "three_stage", 1)      # 1-tile chunks: Bx > 8000
+                assert_parity(got1, x, op, "inclusive", label="3stage K=1")
+
+
 def test_misaligned_and_inplace():
     for op, dt in COMBOS:
         N, G = 12347, 3

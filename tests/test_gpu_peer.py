@@ -133,3 +133,34 @@ def test_peer_two_processes_ipc(tmp_path):
     for r, p in enumerate(procs):
         assert p.returncode == 0, "rank %d failed:\n%s" % (r, logs[r][-3000:])
         assert open(os.path.join(tmp_path, "rank%d" % r)).read().startswith("ok"), logs[r][-2000:]
+
+
+def test_c5_rank_portion_full_size():
+    """configs[4] (N = 2^36 over 8 GPUs) gives every rank a 2^33-element int32 portion
+    (32 GiB in + 32 GiB out).  Here the portion runs at full size as the LAST rank of a
+    W = 2 loopback whose rank 0 holds a 3*2^20 prefix (non-trivial carry through the fused
+    exchange), in the launch configuration bench.py times; every output element is checked
+    against the streaming oracle of the concatenated problem."""
+    from gpu_util import device_inputs
+    import oracle
+    L0, L1 = 3 << 20, 1 << 33
+    seed = 0x5CA2018 + 5
+    comms = multi.PeerComm.loopback(2, 1)
+    try:
+        x0 = device_inputs("i32", L0, seed)
+        x1 = device_inputs("i32", L1, seed, offset=L0)        # the same counter stream, continued
+        y0 = multi.scan_multi(x0, "add", "inclusive", mode="elements", backend="peer", comm=comms[0])
+        y1 = multi.scan_multi(x1, "add", "inclusive", mode="elements", backend="peer", comm=comms[1])
+        torch.cuda.synchronize()
+        so = oracle.StreamAdd(np.int32, "inclusive")
+        assert np.array_equal(to_host(y0, np.int32), so.feed(to_host(x0, np.int32)))
+        del x0, y0
+        step = 1 << 26
+        for a in range(0, L1, step):
+            ref = so.feed(to_host(x1[a:a + step], np.int32))
+            got = to_host(y1[a:a + step], np.int32)
+            assert np.array_equal(got, ref), "c5 rank portion chunk %d" % (a // step)
+    finally:
+        torch.cuda.synchronize()
+        for c in comms:
+            c.close()
