@@ -119,15 +119,25 @@ __device__ __forceinline__ bool peer_last_cta(uint32_t* counter) {
 }
 
 // ------------------------------------------------------------------ Stage 2
+// A round of AUX_ITEMS consecutive chunk values per lane: all loads of a round are issued
+// together (one memory latency per 32*AUX_ITEMS values instead of per 32), scanned
+// serially in registers, then across lanes with shuffles (the tile engine's structure).
+constexpr int AUX_ITEMS = 8;
+
 template <class Op>
 __device__ __forceinline__ void aux_scan_problem(const ChunkParams& p, int64_t g, int lane, bool push) {
     using C = typename Op::Carry;
     uint64_t* a = p.aux + g * p.Bx;
     C run = Op::cidentity();
-    for (int64_t b = 0; b < p.Bx; b += 32) {
-        const int64_t i = b + lane;
-        C v = i < p.Bx ? slot_get<C>(a[i]) : Op::cidentity();
-        C incl = v;
+    for (int64_t b = 0; b < p.Bx; b += 32 * AUX_ITEMS) {
+        const int64_t i0 = b + (int64_t)lane * AUX_ITEMS;
+        C v[AUX_ITEMS];
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) v[k] = i0 + k < p.Bx ? slot_get<C>(a[i0 + k]) : Op::cidentity();
+        C t = Op::cidentity();
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) t = Op::capply(t, v[k]);
+        C incl = t;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
             C y = shfl_up_c<C>(incl, d);
@@ -135,7 +145,12 @@ __device__ __forceinline__ void aux_scan_problem(const ChunkParams& p, int64_t g
         }
         C ex = shfl_up_c<C>(incl, 1);
         if (lane == 0) ex = Op::cidentity();
-        if (i < p.Bx) a[i] = slot_put(Op::capply(run, ex));
+        C r = Op::capply(run, ex);
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) {
+            if (i0 + k < p.Bx) a[i0 + k] = slot_put(r);
+            r = Op::capply(r, v[k]);
+        }
         run = Op::capply(run, shfl_idx_c<C>(incl, 31));
     }
     if (lane == 0) {
@@ -166,10 +181,15 @@ __global__ void __launch_bounds__(WARPS * 32) aux_scan_cta_kernel(ChunkParams p)
     }
     uint64_t* a = p.aux + g * p.Bx;
     C run = Op::cidentity();
-    for (int64_t b = 0; b < p.Bx; b += WARPS * 32) {
-        const int64_t i = b + threadIdx.x;
-        const C v = i < p.Bx ? slot_get<C>(a[i]) : Op::cidentity();
-        C incl = v;
+    for (int64_t b = 0; b < p.Bx; b += WARPS * 32 * AUX_ITEMS) {
+        const int64_t i0 = b + (int64_t)threadIdx.x * AUX_ITEMS;
+        C v[AUX_ITEMS];
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) v[k] = i0 + k < p.Bx ? slot_get<C>(a[i0 + k]) : Op::cidentity();
+        C t = Op::cidentity();
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) t = Op::capply(t, v[k]);
+        C incl = t;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
             C y = shfl_up_c<C>(incl, d);
@@ -180,13 +200,18 @@ __global__ void __launch_bounds__(WARPS * 32) aux_scan_cta_kernel(ChunkParams p)
         C wp = Op::cidentity(), btot = Op::cidentity();
 #pragma unroll 4
         for (int w = 0; w < WARPS; ++w) {
-            const C t = s_w[w];
-            if (w < warp) wp = Op::capply(wp, t);
-            btot = Op::capply(btot, t);
+            const C tw = s_w[w];
+            if (w < warp) wp = Op::capply(wp, tw);
+            btot = Op::capply(btot, tw);
         }
         C ex = shfl_up_c<C>(incl, 1);
         if (lane == 0) ex = Op::cidentity();
-        if (i < p.Bx) a[i] = slot_put(Op::capply(Op::capply(run, wp), ex));
+        C r = Op::capply(Op::capply(run, wp), ex);
+#pragma unroll
+        for (int k = 0; k < AUX_ITEMS; ++k) {
+            if (i0 + k < p.Bx) a[i0 + k] = slot_put(r);
+            r = Op::capply(r, v[k]);
+        }
         run = Op::capply(run, btot);
         __syncthreads();
     }
@@ -363,7 +388,7 @@ cudaError_t launch_maybe_pdl(Kern kern, unsigned blocks, unsigned threads, const
 }
 template <class Op>
 cudaError_t auxscan_op(const ChunkParams& p, cudaStream_t s) {
-    if (p.Bx > 256) {               // many chunks per problem: a CTA per problem
+    if (p.Bx > 32 * AUX_ITEMS) {    // many chunks per problem: a CTA per problem
         if (p.G > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
         return launch_maybe_pdl(aux_scan_cta_kernel<Op, 32>, (unsigned)p.G, 32 * 32, p, s);
     }
