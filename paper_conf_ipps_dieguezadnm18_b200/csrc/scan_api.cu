@@ -46,22 +46,26 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 // from the on-box sweep recorded in profiles/ (bench.py --sweep).
 //   many problems of moderate N (rows 16-byte aligned): the paper's own batch mapping wins
 //     on B200 -- one CTA per problem (cascade, L_y = 1) for N >= 4096, one warp per problem
-//     (L_y = 8) for 1024 <= N < 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
-//   short rows (N < 1024) or unaligned rows: flat segmented look-back, one tile per CTA;
-//   few large problems (G*N >= 2^22): pipelined look-back with 64 KiB tiles;
-//   small totals (latency bound, L2 resident): pipelined look-back with 32 KiB tiles.
-// `aligned` = both base pointers 16-byte aligned.
+//     (L_y = 8) for 768 <= N < 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
+//   short rows (N < 1024, 16-byte aligned base pointers): several whole problems per warp
+//     (packed_warp; power-of-two N <= 512 at ~104 % of copy, ragged N ~85-91 %), against
+//     ~65-78 % for the flat segmented look-back (tools/short_probe.py);
 //   small totals of few problems (<= 2^22 elements, L2 resident, latency bound): the
 //     paper's three-stage form -- three short kernels beat one persistent look-back launch
-//     in device time (configs[0]: ~6 us vs ~7.5 us).
+//     in device time (configs[0]: ~5 us vs ~7.5 us);
+//   everything else (few large problems, unaligned pointers): single-pass look-back
+//     (L2-staged variant for G*N >= 2^22, one-tile-per-CTA for short unaligned rows).
 //   (boundary re-measured with 64-byte descriptor slots, profiles/r01_boundary.txt: the
 //    look-back matches or beats the CTA cascade up to G = 2048; the cascade wins from
 //    G = 4096, where every SM holds many whole problems)
+// `aligned` = both base pointers 16-byte aligned.
 scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
     if (rows_aligned && G >= 4096 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
-    if (rows_aligned && G >= 1184 && N >= 1024 && N < 4096) return SCAN_ALGO_CASCADE_WARP;
+    if (rows_aligned && G >= 1184 && N >= 768 && N < 4096) return SCAN_ALGO_CASCADE_WARP;
     if (G <= 16 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    // short rows: several whole problems per warp (power-of-two N <= 512 flag-free)
+    if (aligned && N < 1024) return SCAN_ALGO_PACKED_WARP;
     return SCAN_ALGO_LOOKBACK;
 }
 int choose_lookback_variant(int64_t N, int64_t G) {
@@ -84,6 +88,30 @@ int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
     // batch kernels do).  ~1184 long chunks spread the concurrent streams ~29 MB apart at
     // 2^33 elements and Stage 3 ran at ~92 % of copy (measured).
     return std::min<int64_t>(chunk, kMaxChunkTiles * tile);
+}
+
+// problems per warp span of the packed kernel.  A span is walked in 1024-element windows,
+// so a span of k*N elements wastes the unused tail of its last window; k is a multiple of
+// q = 4/gcd(N,4) so every span starts 16-byte aligned.  `target` > 0: the largest such k
+// with k*N <= target (at least q).  Default: among spans of 2048..8192 elements the one
+// whose windows are best used (ties: the shortest) -- measured on B200 (tools/short_probe.py):
+// ~4096-element spans beat 1024-element ones by 3-9 % for ragged N, and a half-empty last
+// window costs its full latency.
+constexpr int64_t kPackedMaxN = int64_t(1) << 24;
+constexpr int64_t kPackedWindow = 1024;
+int64_t packed_span_problems(int64_t N, int64_t target) {
+    N = std::max<int64_t>(N, 1);
+    const int64_t q = (N % 4 == 0) ? 1 : (N % 2 == 0) ? 2 : 4;
+    if (target > 0) return std::max<int64_t>(target / N / q * q, q);
+    int64_t best = q;
+    double best_u = -1.0;
+    for (int64_t k = q; k == q || k * N <= 8192; k += q) {
+        const int64_t span = k * N;
+        if (span < 2048 && (k + q) * N <= 8192) continue;
+        const double u = (double)span / (double)(((span + kPackedWindow - 1) / kPackedWindow) * kPackedWindow);
+        if (u > best_u + 1e-9) { best_u = u; best = k; }
+    }
+    return best;
 }
 
 // Look-back workspace: ctl | desc[C] (16-byte slots).  The layout depends only on the
@@ -255,6 +283,13 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         ChunkParams p = chunk_params(in, out, N, G, kind);
         p.chunk = std::max<int64_t>(N, 1); p.Bx = 1;
         return from_cuda(launch_warp_cascade(opcode(op, dt), p, s));
+    }
+    case SCAN_ALGO_PACKED_WARP: {
+        if (N > kPackedMaxN) return SCAN_ERR_UNSUPPORTED;
+        ChunkParams p = chunk_params(in, out, N, G, kind);
+        p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+        p.chunk = packed_span_problems(N, param); p.Bx = 1;
+        return from_cuda(launch_packed_warp(opcode(op, dt), p, s));
     }
     case SCAN_ALGO_THREE_STAGE: {
         void* w = nullptr;
@@ -440,7 +475,7 @@ scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_
                           scan_kind kind, scan_algo algo, int64_t param, void* workspace,
                           size_t workspace_bytes, void* stream) {
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
-    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_THREE_STAGE) return SCAN_ERR_UNSUPPORTED;
+    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_PACKED_WARP) return SCAN_ERR_UNSUPPORTED;
     int64_t total = 0;
     scan_status st = check_shape(N, G, &total);
     if (st != SCAN_OK) return st;

@@ -15,6 +15,8 @@
 //                                                CTA-per-problem batch kernel (L_y = 1).
 //   warp_cascade                                  one WARP per problem, cascade over
 //                                                V*128-element windows (small/medium N).
+//   packed_warp                                   k whole SHORT problems per warp (one
+//                                                span of k*N elements, segmented scan).
 //
 // Aux, totals and carry slots are 8 bytes: the 32-bit value in the low half, or the fp64
 // carry of f32 add.  All problem-local indices are 64-bit (N*G reaches 2^36).
@@ -351,6 +353,111 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
     }
 }
 
+// ------------------------------------------------------------------ packed short problems
+// Several whole problems per warp (L_x < 32 threads per problem): warp w owns
+// problems [w*k, (w+1)*k) -- one contiguous span of k*N elements that starts and ends on
+// problem boundaries, 16-byte aligned (k*N % 4 == 0, chosen on the host) -- and walks it in
+// V*128-element windows with a SEGMENTED scan (heads every N elements).  No carry crosses
+// a span, so there is no inter-warp dependency at all; inside the span the segmented carry
+// runs from window to window (a head resets it).
+template <class Op, int WARPS, int V, bool EXCL>
+__global__ void __launch_bounds__(WARPS * 32) packed_warp_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t k = p.chunk;                       // problems per span
+    const int64_t g0 = ((int64_t)blockIdx.x * WARPS + warp) * k;
+    if (g0 >= p.G) return;
+    const int64_t base = g0 * p.N;
+    const int64_t end = min(g0 + k, p.G) * p.N;
+    const T* in = (const T*)p.in;
+    T* out = (T*)p.out;
+    const uint32_t N32 = (uint32_t)p.N;
+    C carry = Op::cidentity();                       // segmented: value since the last head
+    for (int64_t off = base; off < end; off += WCH) {
+        Row4<T> x[V];                                // the whole window in flight at once
+#pragma unroll
+        for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, off + j * 128 + lane * 4, end, p.vec);
+        // then row by row: only the running carry lives across rows (few registers)
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            const unsigned hd = row_heads_small((uint32_t)(off - base) + j * 128 + lane * 4, 0u, N32);
+            T v = row_reduce<Op, true>(x[j], hd);
+            const unsigned hm = __ballot_sync(FULL, hd != 0u);
+            T lin; bool lfl;
+            T incl = warp_seg_scan<Op, true>(v, hm, lin, lfl);
+            T rt = shfl_idx<T>(incl, 31);
+            store_row<Op>(out, off + j * 128 + lane * 4, end, p.vec,
+                          row_output<Op, true, EXCL>(x[j], hd, lin, lfl, Op::from_carry(carry)));
+            carry = hm ? Op::to_carry(rt) : Op::capply(carry, Op::to_carry(rt));
+        }
+    }
+}
+
+// Power-of-two N <= 512 (the paper's problem sizes): every V*128-element
+// window of the flat array holds whole problems, so warp w simply owns window w and the
+// segment structure is regular -- no head flags, no ballots:
+//   N <= 4        a problem lies inside one lane's 4-element row: serial, resets in-lane;
+//   8 <= N <= 128 a problem spans L = N/4 lanes: sub-warp scan (shfl.up, segments of L);
+//   N >= 256      a problem spans R = N/128 rows: full-warp scan per row, the row carry
+//                 resets every R rows.
+template <class Op>
+__device__ __forceinline__ typename Op::T shfl_up_w(typename Op::T v, int d, int width) {
+    return from_bits<typename Op::T>(__shfl_up_sync(FULL, to_bits<typename Op::T>(v), d, width));
+}
+template <class Op, int WARPS, int V, bool EXCL>
+__global__ void __launch_bounds__(WARPS * 32) packed_pow2_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t base = ((int64_t)blockIdx.x * WARPS + warp) * WCH;
+    const int64_t total = p.N * p.G;
+    if (base >= total) return;
+    const T* in = (const T*)p.in;
+    T* out = (T*)p.out;
+    const int n = (int)p.N;
+    Row4<T> x[V];
+#pragma unroll
+    for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, base + j * 128 + lane * 4, total, p.vec);
+    if (n <= 4) {
+        const unsigned hd = n == 1 ? 0xFu : n == 2 ? 0x5u : 0x1u;
+#pragma unroll
+        for (int j = 0; j < V; ++j)
+            store_row<Op>(out, base + j * 128 + lane * 4, total, p.vec,
+                          row_output<Op, true, EXCL>(x[j], hd, Op::identity(), true, Op::identity()));
+    } else if (n <= 128) {
+        const int L = n >> 2;                       // lanes per problem
+        const int sl = lane & (L - 1);              // lane index inside its problem
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            T v = row_reduce<Op, false>(x[j], 0u);
+            for (int d = 1; d < L; d <<= 1) {
+                T y = shfl_up_w<Op>(v, d, L);
+                if (sl >= d) v = Op::apply(y, v);
+            }
+            T e = shfl_up_w<Op>(v, 1, L);
+            if (sl == 0) e = Op::identity();
+            store_row<Op>(out, base + j * 128 + lane * 4, total, p.vec,
+                          row_output<Op, false, EXCL>(x[j], 0u, e, false, Op::identity()));
+        }
+    } else {
+        const int R = n >> 7;                       // rows per problem (2 or 4)
+        T run = Op::identity();
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+            T v = row_reduce<Op, false>(x[j], 0u);
+            T e; bool ef;
+            T incl = warp_seg_scan<Op, false>(v, 0u, e, ef);
+            T rt = shfl_idx<T>(incl, 31);
+            if ((j & (R - 1)) == 0) run = Op::identity();
+            store_row<Op>(out, base + j * 128 + lane * 4, total, p.vec,
+                          row_output<Op, false, EXCL>(x[j], 0u, Op::apply(run, e), false, Op::identity()));
+            run = Op::apply(run, rt);
+        }
+    }
+}
+
 // fused exchange, empty local portion: wait for ranks < rank, acknowledge them
 __global__ void peer_ack_kernel(PeerParams pp) {
     if (threadIdx.x != 0) return;
@@ -410,6 +517,27 @@ cudaError_t warp_op(const ChunkParams& p, cudaStream_t s) {
     warp_cascade_kernel<Op, WC_WARPS, WC_V><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
     return cudaGetLastError();
 }
+template <class Op>
+cudaError_t packed_op(const ChunkParams& p, cudaStream_t s) {
+    const bool pow2 = p.N > 0 && p.N <= 512 && (p.N & (p.N - 1)) == 0;
+    if (pow2 && p.vec) {                                   // regular segments, one window per warp
+        constexpr int WCH = WC_V * 128;
+        const int64_t windows = (p.N * p.G + WCH - 1) / WCH;
+        const int64_t blocks = (windows + WC_WARPS - 1) / WC_WARPS;
+        if (blocks == 0) return cudaSuccess;
+        if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+        if (p.exclusive) packed_pow2_kernel<Op, WC_WARPS, WC_V, true><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
+        else packed_pow2_kernel<Op, WC_WARPS, WC_V, false><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
+        return cudaGetLastError();
+    }
+    const int64_t spans = (p.G + p.chunk - 1) / p.chunk;
+    const int64_t blocks = (spans + WC_WARPS - 1) / WC_WARPS;
+    if (blocks == 0) return cudaSuccess;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    if (p.exclusive) packed_warp_kernel<Op, WC_WARPS, WC_V, true><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
+    else packed_warp_kernel<Op, WC_WARPS, WC_V, false><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
 
 #define SCANB200_DISPATCH(fn)                                          \
     switch (op) {                                                      \
@@ -430,6 +558,7 @@ cudaError_t launch_chunk_reduce(OpCode op, const ChunkParams& p, cudaStream_t s)
 cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(auxscan_op) }
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(scan_op) }
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_op) }
+cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(packed_op) }
 cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s) {
     if (!pp.on || pp.rank == 0) return cudaSuccess;
     peer_ack_kernel<<<1, 32, 0, s>>>(pp);

@@ -92,6 +92,9 @@ cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 // Warp-per-problem cascade (L_y = warps per block problems per CTA).
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Packed short problems: p.chunk = k whole problems per warp span (k*N % 4 == 0 when
+// p.vec), segmented scan, no carry between spans (L_x < 32).
+cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s);
 // Fused exchange with an empty local portion (no Stage 3 CTAs): one CTA waits for the
 // flags of ranks < rank and acknowledges them, so peers never wait on this rank.
 cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s);

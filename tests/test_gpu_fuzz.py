@@ -17,11 +17,12 @@ pytestmark = pytest.mark.gpu
 @pytest.mark.parametrize("seed", range(6))
 def test_random_cases(seed):
     rng = random.Random(2018 + seed)
-    algos = [("auto", -1), ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0), ("three_stage", 3)] + \
+    algos = [("auto", -1), ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0), ("three_stage", 3),
+             ("packed_warp", -1), ("packed_warp", 300)] + \
             [("lookback", v) for v in range(_lib.lib_num_lookback_variants())]
     for case in range(40):
         N = rng.choice([rng.randint(1, 300), rng.randint(300, 20000), rng.randint(20000, 400000)])
-        G = rng.choice([1, 1, 2, rng.randint(1, 40)])
+        G = rng.choice([1, 1, 2, rng.randint(1, 40), rng.randint(100, 5000)])
         if N * G > 3_000_000:
             G = max(1, 3_000_000 // N)
         op, dt = rng.choice(COMBOS)

@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 NS = [1, 2, 3, 4, 5, 7, 31, 32, 33, 127, 128, 129, 511, 513, 1023, 1024, 1025, 4095, 4096, 4097,
       8191, 8192, 8193, 16383, 16385, 3 * 8192 + 5, 100003]
 GS = [1, 2, 3, 7]
-ALGOS = ["lookback", "cascade_cta", "cascade_warp", "three_stage"]
+ALGOS = ["lookback", "cascade_cta", "cascade_warp", "three_stage", "packed_warp"]
 
 
 def _run(x, op, kind, algo="auto", param=-1):
@@ -288,3 +288,24 @@ def test_error_paths():
     h = np.zeros(100, np.int32)
     rc = _lib.lib.scan_batch(h.ctypes.data, h.ctypes.data, 100, 1, 0, 0, 0, None)
     assert rc == 1                                              # host pointer -> INVALID_ARG
+
+
+@pytest.mark.parametrize("param", [-1, 100, 4096])
+def test_packed_short_rows(param):
+    # several whole short problems per warp (segmented spans, PAPER.md:98 L_x < 32): every
+    # residue of N mod 4 (span alignment), spans shorter / longer than one window, ragged G
+    for op, dt in COMBOS:
+        for N in [1, 2, 3, 5, 17, 64, 100, 255, 256, 257, 511, 1000, 1023, 1030]:
+            G = 150001 // N + 3
+            x = inputs.generate(DIST[dt], N * G, seed=N * 31 + G).reshape(G, N)
+            for kind in ("inclusive", "exclusive"):
+                got = _run(x, op, kind, "packed_warp", param)
+                assert_parity(got, x, op, kind, label="packed p=%d %s %s %s N=%d" % (param, op, dt, kind, N))
+
+
+def test_auto_short_rows_use_packed():
+    x = torch.zeros((4096, 300), dtype=torch.int32, device="cuda")
+    assert sb.plan(x)[0] == "packed_warp"
+    assert sb.plan(x[:, :1].contiguous().view(4096, 1))[0] == "packed_warp"
+    y = torch.zeros((4096, 1000), dtype=torch.int32, device="cuda")
+    assert sb.plan(y)[0] == "cascade_warp"
