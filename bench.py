@@ -50,6 +50,35 @@ def _peaks():
     return 6650.0, "fallback (B200_PROFILING.md)", {}
 
 
+# ---------------------------------------------------------------- multi-rank plumbing
+# SCANB200_BENCH_BACKEND=gloo + SCANB200_BENCH_ONE_GPU=1 run every rank on cuda:0 with a gloo
+# process group: a dry run of the multi-rank control flow (barriers, max over ranks, the
+# peer-memory exchange between processes) on a one-GPU box; NCCL refuses two ranks on one GPU.
+DIST_BACKEND = os.environ.get("SCANB200_BENCH_BACKEND", "nccl")
+ONE_GPU = os.environ.get("SCANB200_BENCH_ONE_GPU") == "1"
+
+
+def max_over_ranks(v: float, world: int) -> float:
+    if world == 1:
+        return v
+    dev = "cuda" if DIST_BACKEND == "nccl" else "cpu"
+    t = torch.tensor([v], dtype=torch.float64, device=dev)
+    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    return float(t.item())
+
+
+def all_gather_totals(t: torch.Tensor, world: int) -> torch.Tensor:
+    """[W, G] totals of all ranks (the torch-backend exchange of the phase breakdown)."""
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    if world == 1:
+        return t.view(1, -1)
+    if DIST_BACKEND == "nccl":
+        return multi.exchange_totals(t)
+    parts = [torch.empty_like(t, device="cpu") for _ in range(world)]
+    torch.distributed.all_gather(parts, t.cpu())
+    return torch.stack(parts).to(t.device)
+
+
 # ---------------------------------------------------------------- clocks during the timed region
 class ClockSampler:
     def __init__(self, dev_index: int):
@@ -156,8 +185,10 @@ def kernel_times(sb, xs, outs, reps):
     return res
 
 
-def e2e(sb, K=3):
-    """The same step through the public host-buffer API: pinned host in -> scan -> host out."""
+def e2e(sb, world=1, K=3):
+    """The same step through the public host-buffer API: pinned host in -> scan -> host out.
+    Under torchrun every rank runs it at once on its own GPU (its own PCIe link); the time
+    is the max over ranks and the value counts the elements of all ranks."""
     import inputs
     hin, hout = {}, []
     for dt in ("i32", "f32"):
@@ -172,14 +203,82 @@ def e2e(sb, K=3):
         for i, (dt, op, kind) in enumerate(VARIANTS):
             sb.scan_host(hin[dt], op, kind, out=hout[i].view(NPDT[dt]))
     one()
+    if world > 1:
+        torch.distributed.barrier()
     t0 = time.perf_counter()
     for _ in range(K):
         one()
     dt_s = (time.perf_counter() - t0) / K
+    dt_s = max_over_ranks(dt_s, world)
     elems = len(VARIANTS) * G_C2 * N_C2
-    return {"value": elems / dt_s / 1e9, "unit": "Gelem/s", "ms_per_step": dt_s * 1e3, "steps": K,
-            "h2d_bytes_per_step": elems * 4, "d2h_bytes_per_step": elems * 4,
-            "api": "scan_batch_host (pinned host buffers, library-pipelined H2D/scan/D2H)"}
+    res = {"value": world * elems / dt_s / 1e9, "unit": "Gelem/s", "ms_per_step": dt_s * 1e3, "steps": K,
+           "h2d_bytes_per_step": elems * 4, "d2h_bytes_per_step": elems * 4,
+           "api": "scan_batch_host (pinned host buffers, library-pipelined H2D/scan/D2H)",
+           "timing": "host wall clock around the synchronous calls, max over ranks"}
+    res["pcie_ceiling"] = pcie_ceiling(elems * 4)
+    res["frac_of_pcie_ceiling"] = (elems / dt_s / 1e9) / res["pcie_ceiling"]["Gelem/s_ceiling"]
+    return res
+
+
+def pcie_ceiling(nbytes: int, reps: int = 3):
+    """Context for e2e: plain torch pinned-memory copies of the step's bytes, H2D and D2H
+    at the same time on two streams (what any host-buffer scan must move)."""
+    h_in = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    h_out = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d_in = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d_out = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+
+    def both():
+        with torch.cuda.stream(s1):
+            d_in.copy_(h_in, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h_out.copy_(d_out, non_blocking=True)
+        torch.cuda.synchronize()
+    both()
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        both()
+    dt_s = (time.perf_counter() - t0) / reps
+    gbs = nbytes / dt_s / 1e9
+    del d_in, d_out
+    torch.cuda.empty_cache()
+    return {"GB/s_each_way": gbs, "Gelem/s_ceiling": gbs / 4,
+            "how": "torch pinned H2D + D2H copies of %d bytes each, concurrently on two streams" % nbytes}
+
+
+def c4_problems(sb, dev, world, rank, reps=5):
+    """configs[3]: G = 2^16 problems of N = 2^16 int32 sharded by problem (Case 1,
+    PAPER.md:191-193): rank r scans problems [floor(rG/W), floor((r+1)G/W)), no
+    collective.  Strong scaling (the total is fixed); at W = 1 the whole 16 GiB batch."""
+    import inputs
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    G, N = 1 << 16, 1 << 16
+    g0, g1 = multi.partition(G, world, rank)
+    x = torch.empty((g1 - g0) * N, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "i32", SEED + 4, offset=g0 * N)
+    x = x.view(g1 - g0, N)
+    y = torch.empty_like(x)
+    for _ in range(2):
+        multi.scan_multi(x, "add", "inclusive", mode="problems", out=y)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    for _ in range(reps):
+        multi.scan_multi(x, "add", "inclusive", mode="problems", out=y)
+    s1.record()
+    torch.cuda.synchronize()
+    ms = max_over_ranks(s0.elapsed_time(s1) / reps, world)
+    hbm, _, _ = _peaks()
+    per_gpu_gbs = 8.0 * G * N / world / (ms * 1e-3) / 1e9
+    kern = "%s %s" % sb.plan(x, y)
+    del x, y
+    torch.cuda.empty_cache()
+    return {"G": G, "N": N, "problems_per_gpu": G // world, "ms": ms, "Gelem/s": G * N / ms / 1e6,
+            "per_gpu_GB/s": per_gpu_gbs, "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
+            "scaling": "strong (fixed 2^32-element batch)", "kernel": kern}
 
 
 # ---------------------------------------------------------------- CPU oracle (reference arm / baseline)
@@ -291,7 +390,8 @@ def extras(sb, dev):
     return out
 
 
-def elements_mode(sb, dev, world, rank, n_local=1 << 33, reps=10):
+def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB200_BENCH_ELEMS_LOG2", "33")),
+                  reps=10):
     """configs[4]: one int32 add-scan sharded by elements (Multi-GPU Problem Scattering,
     PAPER.md:195-205): each rank owns a contiguous 2^33-element portion (32 GiB in + 32 GiB
     out) of ONE problem -- at W = 8 the problem is configs[4]'s N = 2^36.  Stage 1+2 ->
@@ -305,7 +405,7 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 33, reps=10):
     # the fused exchange (Stage 2 pushes the totals into later ranks' HBM, Stage 3 waits on
     # the device; no collective call) is the product path; NCCL all-gather beside it
     comms = {"peer": multi.PeerComm(1) if world > 1 else multi.PeerComm.loopback(1, 1)[0]}
-    if world > 1:
+    if world > 1 and DIST_BACKEND == "nccl":
         comms["nccl"] = multi.NativeComm()
 
     def run(name):
@@ -324,12 +424,7 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 33, reps=10):
             run(name)
         s1.record()
         torch.cuda.synchronize()
-        ms = s0.elapsed_time(s1) / reps
-        if world > 1:
-            t = torch.tensor([ms], device=dev)
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            ms = float(t.item())
-        times[name] = ms
+        times[name] = max_over_ranks(s0.elapsed_time(s1) / reps, world)
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
@@ -346,7 +441,7 @@ def elements_mode(sb, dev, world, rank, n_local=1 << 33, reps=10):
         ev[0].record()
         sb.shard_totals(x, "add", totals=t)
         ev[1].record()
-        allt = multi.exchange_totals(t) if world > 1 else t.view(1, -1)
+        allt = all_gather_totals(t, world)
         ev[2].record()
         sb.shard_scan(x, allt, rank, world, "add", "inclusive", out=y)
         ev[3].record()
@@ -453,11 +548,16 @@ def main():
         return
 
     import paper_conf_ipps_dieguezadnm18_b200 as sb
+    if ONE_GPU:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if DIST_BACKEND == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(DIST_BACKEND)
     if args.sweep:
         rows = sweep(sb, dev)
         if rank == 0:
@@ -477,19 +577,28 @@ def main():
         total_ms, _ = timed_steps(sb, xs, outs, args.steps)
     if world > 1:
         torch.distributed.barrier()
-        t = torch.tensor([total_ms], device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        total_ms = float(t.item())
-    # average launch duration of each scan kernel: `reps` back-to-back launches of the same
-    # call between two events on the launching stream (no events between launches)
+        total_ms = max_over_ranks(total_ms, world)
+    # average launch duration of the dominant kernel, live over the timed region: every
+    # launch in it is the same kernel family on the same bytes (the plan is checked below),
+    # so it is the timed region's device time / its launches.  Events between launches are
+    # avoided on purpose: an event pair around each ~85 us launch adds ~2 us of gap (measured).
+    # Per-variant averages (reps back-to-back launches of one call between two events on the
+    # launching stream) are reported beside it.
     launch_ms = kernel_times(sb, xs, outs, max(20, args.steps // 4))
+    plans = {sb.plan(xs[dt], outs[i]) for i, (dt, _, _) in enumerate(VARIANTS)}
+    live_launch_ms = total_ms / (args.steps * len(VARIANTS))
 
     ms_step = total_ms / args.steps
     elems_step = len(VARIANTS) * G_C2 * N_C2 * world
     value = elems_step / (ms_step * 1e-3) / 1e9
     bytes_launch = 2 * 4 * G_C2 * N_C2
     dom = max(range(len(VARIANTS)), key=lambda i: launch_ms[i])
-    achieved = bytes_launch / (launch_ms[dom] * 1e-3) / 1e9
+    if len(plans) == 1:
+        achieved, dom_ms, timing = (bytes_launch / (live_launch_ms * 1e-3) / 1e9, live_launch_ms,
+                                    "timed region device time / launches (all launches are this kernel)")
+    else:
+        achieved, dom_ms, timing = (bytes_launch / (launch_ms[dom] * 1e-3) / 1e9, launch_ms[dom],
+                                    "back-to-back launches of the slowest variant between two events")
     algo, param = sb.plan(xs[VARIANTS[dom][0]], outs[dom])
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -509,10 +618,11 @@ def main():
                      "frac": achieved / hbm, "traffic": traffic,
                      "kernel": "%s [algo=%s param=%d] on %s %s %s" % (
                          sb.KERNEL_NAMES[algo], algo, param, *VARIANTS[dom]),
-                     "bytes_per_launch": bytes_launch, "ms_per_launch": launch_ms[dom],
+                     "bytes_per_launch": bytes_launch, "ms_per_launch": dom_ms, "timing": timing,
                      "bytes_basis": "2 x 4 B x G x N (read input once, write output once)",
                      "peak_src": hbm_src + " copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"},
         "per_launch_ms": {"%s_%s_%s" % v: m for v, m in zip(VARIANTS, launch_ms)},
+
         "gpu_launches": len(VARIANTS) * args.steps,
         "clocks": clk.summary(),
     }
@@ -520,8 +630,9 @@ def main():
         el = elements_mode(sb, dev, world, rank)
         res["elements_mode_sharded_problem"] = el
         torch.cuda.empty_cache()
-    if rank == 0 and not args.no_e2e:
-        res["e2e"] = e2e(sb)
+        res["c4_problems_mode"] = c4_problems(sb, dev, world, rank)
+    if not args.no_e2e:
+        res["e2e"] = e2e(sb, world)
     if rank == 0 and world == 1 and not args.no_cpu:
         res["cpu_baseline"] = cpu_oracle_rate()
     if rank == 0 and world == 1 and not args.no_extras:
