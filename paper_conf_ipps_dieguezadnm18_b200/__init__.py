@@ -147,7 +147,8 @@ KERNEL_NAMES = {"lookback": "lookback_*_kernel (decoupled look-back)",
                 "cascade_cta": "chunk_scan_kernel (one CTA per problem, cascade)",
                 "cascade_warp": "warp_cascade_kernel (one warp per problem, cascade)",
                 "three_stage": "chunk_reduce + aux_scan + chunk_scan kernels",
-                "packed_warp": "packed_warp_kernel (k short problems per warp, segmented)"}
+                "packed_warp": "packed_warp_kernel (k short problems per warp, segmented)",
+                "cluster": "cluster_scan_kernel (one thread-block cluster per problem, DSMEM aggregates)"}
 
 
 def plan(x: torch.Tensor, out: torch.Tensor | None = None) -> tuple[str, int]:

@@ -63,6 +63,12 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
     if (rows_aligned && G >= 4096 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
     if (rows_aligned && G >= 1184 && N >= 768 && N < 4096) return SCAN_ALGO_CASCADE_WARP;
+    // few short / medium problems (latency bound, tools/cluster_probe.py on B200,
+    // profiles/r01_cluster_probe.jsonl): one CTA per problem up to 8192 elements
+    // (~2.5-3.3 us per call against 5-12 us for three-stage / look-back), one thread-block
+    // cluster per problem (DSMEM aggregates) up to 2^15 (2^16 for G <= 4): ~3.7-4.6 us
+    if (G <= 148 && N <= 8192) return SCAN_ALGO_CASCADE_CTA;
+    if ((G <= 64 && N <= 32768) || (G <= 4 && N <= 65536)) return SCAN_ALGO_CLUSTER;
     if (G <= 16 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     // short rows: several whole problems per warp (power-of-two N <= 512 flag-free)
     if (aligned && N < 1024) return SCAN_ALGO_PACKED_WARP;
@@ -74,11 +80,32 @@ int choose_lookback_variant(int64_t N, int64_t G) {
     return total >= (int64_t(1) << 22) ? 3 : 1;
 }
 
+// cluster family: param = 32 * variant + csize (csize a power of two <= 16), < 0 = auto:
+// 4096-element tiles (variant 1), the smallest cluster that covers the problem in one
+// round (<= 16) -- the measured best for 2^13 < N <= 2^16 at G = 1..16
+void cluster_config(int64_t N, int64_t param, int* variant, int* csize) {
+    if (param >= 0) {
+        *variant = (int)((param / 32) % 3);
+        int c = (int)(param % 32);
+        int q = 1;
+        while (q < c && q < kMaxClusterCtas) q <<= 1;
+        *csize = q;
+        return;
+    }
+    *variant = 1;
+    const int64_t tiles = (N + cluster_tile_elems(1) - 1) / cluster_tile_elems(1);
+    int q = 1;
+    while (q < tiles && q < kMaxClusterCtas) q <<= 1;
+    *csize = q;
+}
+
 int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
     const int64_t tile = chunk_tile_elems();
     if (K > 0) return K * tile;
-    // latency-bound totals (configs[0]): two tiles per chunk measured best on B200
-    // (2^20: 5.1 us at K = 2 against 5.9 us at K = 1 and 6.6 us at K = 3, CUDA graph)
+    // latency-bound totals: one tile per chunk up to 2^19 elements (G = 1: 4.9-5.1 us
+    // against 5.6-5.7 us at K = 2), two tiles up to 2^22 (configs[0], 2^20: 5.5 us against
+    // 5.7 us at K = 1); tools/g1_probe.py, profiles/r01_g1_probe.jsonl
+    if (N * G <= (int64_t(1) << 19)) return tile;
     if (N * G <= (int64_t(1) << 22)) return 2 * tile;
     int64_t bx = std::max<int64_t>(1, (kTargetCtas + G - 1) / G);
     int64_t chunk = (N + bx - 1) / bx;
@@ -291,6 +318,13 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         p.chunk = packed_span_problems(N, param); p.Bx = 1;
         return from_cuda(launch_packed_warp(opcode(op, dt), p, s));
     }
+    case SCAN_ALGO_CLUSTER: {
+        int variant = 0, csize = 0;
+        cluster_config(N, param, &variant, &csize);
+        if ((int64_t)G * csize > 0x7FFFFFFFll) return SCAN_ERR_UNSUPPORTED;
+        ChunkParams p = chunk_params(in, out, N, G, kind);
+        return from_cuda(launch_cluster_scan(opcode(op, dt), p, variant, csize, s));
+    }
     case SCAN_ALGO_THREE_STAGE: {
         void* w = nullptr;
         size_t wb = 0;
@@ -475,7 +509,7 @@ scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_
                           scan_kind kind, scan_algo algo, int64_t param, void* workspace,
                           size_t workspace_bytes, void* stream) {
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
-    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_PACKED_WARP) return SCAN_ERR_UNSUPPORTED;
+    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_CLUSTER) return SCAN_ERR_UNSUPPORTED;
     int64_t total = 0;
     scan_status st = check_shape(N, G, &total);
     if (st != SCAN_OK) return st;

@@ -95,6 +95,13 @@ cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s)
 // Packed short problems: p.chunk = k whole problems per warp span (k*N % 4 == 0 when
 // p.vec), segmented scan, no carry between spans (L_x < 32).
 cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s);
+// Cluster per problem (scan_cluster.cu): G clusters of csize CTAs (power of two <= 16);
+// the CTAs of one problem exchange their tile aggregates through distributed shared
+// memory (one cluster barrier per round of csize tiles).  variant 0/1/2 = 8192/4096/16384-
+// element tiles.
+constexpr int kMaxClusterCtas = 16;
+int64_t cluster_tile_elems(int variant);
+cudaError_t launch_cluster_scan(OpCode op, const ChunkParams& p, int variant, int csize, cudaStream_t s);
 // Fused exchange with an empty local portion (no Stage 3 CTAs): one CTA waits for the
 // flags of ranks < rank and acknowledges them, so peers never wait on this rank.
 cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s);

@@ -32,7 +32,8 @@
 // Other variants (kept measurable through scan_batch_ex `param`): 1 = 32 KiB tiles,
 // 2 = one tile per CTA (short / unaligned rows), 3 = L2-staged two-read form (limited by
 // L2 slice throughput on B200), 4 = two look-back warps, 5 = register-resident waiting
-// tiles.
+// tiles, 10-12 = one register tile per CTA, 13/14 = thread-block clusters of 16/8 register
+// tiles that combine through DSMEM and look back per cluster (G = 1; G > 1 runs 10).
 //
 // Descriptors (one per tile; reset-free thanks to a 30-bit epoch tag in every word):
 //   word = payload32 << 32 | tag << 2 | status      status 0 X (not ready), 1 A, 2 P
@@ -42,8 +43,12 @@
 //   self-contained, so relaxed (.STRONG.GPU, L1-bypassing) accesses suffice.
 // The last CTA to finish resets the ticket / done counters and advances the epoch, so
 // consecutive launches (also CUDA-graph replays) need no memset.
+#include <cooperative_groups.h>
+
 #include "scan_common.cuh"
 #include "scan_internal.h"
+
+namespace cg = cooperative_groups;
 
 namespace scanb200 {
 
@@ -1165,6 +1170,60 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackPa
     if (threadIdx.x == 0) epilogue(p);
 }
 
+// ---------------------------------------------------------------- clustered look-back
+// One problem (G = 1) of a few 2^20 elements, latency bound (configs[0]).  CS CTAs of one
+// register tile each form a thread-block cluster; the cluster first combines its CTA
+// aggregates through distributed shared memory (one cluster barrier), then only the
+// CLUSTER takes part in the decoupled look-back: descriptor q is cluster q's aggregate /
+// inclusive prefix, so 2^20 elements need 8 descriptors (one look-back round trip) instead
+// of 128.  Clusters follow blockIdx (in-order dispatch).  Every CTA's last warp runs the
+// (identical) look-back itself, so no second cluster barrier is needed; rank 0 publishes.
+template <class Op, int WARPS, int V, int CS>
+__global__ void __launch_bounds__(WARPS * 32) lookback_cluster_kernel(LookbackParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
+    __shared__ T s_wval[WARPS];
+    __shared__ C s_agg, s_carry;
+    cg::cluster_group cl = cg::this_cluster();
+    const unsigned crank = cl.block_rank();
+    const int64_t q = (int64_t)blockIdx.x / CS;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const uint32_t tag = read_tag(p);
+    const int64_t wb = (int64_t)blockIdx.x * TILE + warp * WCH;
+    WarpTile<Op, false, V> wt;
+    wt.load((const T*)p.in, wb, p.total, p.vec);
+    wt.scan();
+    if (lane == 0) s_wval[warp] = wt.wtot;
+    __syncthreads();
+    T wp = Op::identity();
+#pragma unroll
+    for (int w = 0; w < WARPS; ++w)
+        if (w < warp) wp = Op::apply(wp, s_wval[w]);
+    if (warp == WARPS - 1 && lane == 0) s_agg = Op::to_carry(Op::apply(wp, wt.wtot));
+    cl.sync();
+    C a = Op::cidentity();
+    if (lane < CS) a = *cl.map_shared_rank(&s_agg, (unsigned)lane);
+    const C pre = warp_reduce_carry<Op>((unsigned)lane < crank ? a : Op::cidentity());
+    // done with the peers' shared memory: arrive now, wait before exiting
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    if (warp == WARPS - 1) {
+        const C ctot = warp_reduce_carry<Op>(a);
+        if (crank == 0 && lane == 0) Desc<Op>::publish(p, q, tag, q == 0 ? ST_P : ST_A, ctot);
+        C carry = Op::cidentity();
+        if (q > 0) carry = look_back<Op>(p, q, tag);
+        if (lane == 0) {
+            if (crank == 0 && q > 0) Desc<Op>::publish(p, q, tag, ST_P, Op::capply(carry, ctot));
+            s_carry = carry;
+        }
+    }
+    __syncthreads();
+    wt.store((T*)p.out, wb, p.total, p.vec, wp, false, Op::from_carry(Op::capply(s_carry, pre)), p.exclusive);
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+    __syncthreads();
+    if (threadIdx.x == 0) epilogue(p);
+}
+
 // ---------------------------------------------------------------- launchers
 int g_num_sms = 0;
 
@@ -1226,6 +1285,34 @@ cudaError_t launch_regtile(const LookbackParams& p, cudaStream_t s) {
     return cudaGetLastError();
 }
 
+template <class Op, int WARPS, int V, int CS>
+cudaError_t launch_lb_cluster(const LookbackParams& p, cudaStream_t s) {
+    if (p.N != p.total) return launch_regtile<Op, WARPS, V>(p, s);   // G > 1: per-tile look-back
+    constexpr int TILE = WARPS * 32 * V * 4;
+    auto kern = lookback_cluster_kernel<Op, WARPS, V, CS>;
+    static bool init = false;
+    if (!init) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (e != cudaSuccess) return e;
+        init = true;
+    }
+    const int64_t tiles = (p.total + TILE - 1) / TILE;
+    const int64_t grid = (tiles + CS - 1) / CS * CS;
+    if (grid > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid, 1, 1);
+    cfg.blockDim = dim3(WARPS * 32, 1, 1);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = CS;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, p);
+}
+
 template <class Op, int WARPS, int V, int S, int M, int NLB, int PF = 0>
 cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
@@ -1265,6 +1352,8 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 10: return launch_regtile<Op, 16, 4>(p, s);               // one 8192-element register tile per CTA
     case 11: return launch_regtile<Op, 8, 4>(p, s);                // one 4096-element register tile per CTA
     case 12: return launch_regtile<Op, 32, 4>(p, s);               // one 16384-element register tile per CTA
+    case 13: return launch_lb_cluster<Op, 16, 4, 16>(p, s);        // 16-CTA clusters of 8192-element tiles (G = 1)
+    case 14: return launch_lb_cluster<Op, 16, 4, 8>(p, s);         // 8-CTA clusters of 8192-element tiles (G = 1)
     default: return launch_pipelined<Op, 16, 8, 3, 5, 1, 0>(p, s); // as 0 without the L2 prefetch
     }
 }
@@ -1275,7 +1364,7 @@ int64_t lookback_tile_elems(int variant) {
     return (variant == 0 || variant == 4 || variant == 9 || variant == 12) ? 16384 : variant == 5 ? 12288
          : variant == 8 ? 18432 : (variant == 6 || variant == 7 || variant == 11) ? 4096 : 8192;
 }
-int lookback_num_variants() { return 13; }
+int lookback_num_variants() { return 15; }
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

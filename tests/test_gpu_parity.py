@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 NS = [1, 2, 3, 4, 5, 7, 31, 32, 33, 127, 128, 129, 511, 513, 1023, 1024, 1025, 4095, 4096, 4097,
       8191, 8192, 8193, 16383, 16385, 3 * 8192 + 5, 100003]
 GS = [1, 2, 3, 7]
-ALGOS = ["lookback", "cascade_cta", "cascade_warp", "three_stage", "packed_warp"]
+ALGOS = ["lookback", "cascade_cta", "cascade_warp", "three_stage", "packed_warp", "cluster"]
 
 
 def _run(x, op, kind, algo="auto", param=-1):
@@ -39,7 +39,7 @@ def test_shapes_all_algos(algo, op, dt, kind):
             assert_parity(got, x, op, kind, label="%s %s %s %s N=%d G=%d" % (algo, op, dt, kind, N, G))
 
 
-@pytest.mark.parametrize("variant", range(13))
+@pytest.mark.parametrize("variant", range(15))
 def test_lookback_variants(variant):
     for op, dt in COMBOS:
         for N, G in [(1, 3000), (3, 5000), (100, 333), (8193, 5), (65536 + 17, 3), (1 << 20, 1)]:
@@ -47,6 +47,20 @@ def test_lookback_variants(variant):
             for kind in ("inclusive", "exclusive"):
                 got = _run(x, op, kind, "lookback", variant)
                 assert_parity(got, x, op, kind, label="v%d %s %s N=%d G=%d" % (variant, op, dt, N, G))
+
+
+@pytest.mark.parametrize("variant", range(3))
+def test_cluster_sizes(variant):
+    # every cluster size (1..16 CTAs, DSMEM aggregate exchange), one round and several
+    # rounds of csize tiles (register carry between rounds), ragged tails, G > 1
+    for csize in (1, 2, 4, 8, 16):
+        for op, dt in COMBOS:
+            for N, G in [(5, 3), (4096 * csize - 3, 2), (16384 * csize + 4097, 1), (100003, 3)]:
+                x = inputs.generate(DIST[dt], N * G, seed=N + 31 * G + csize).reshape(G, N)
+                for kind in ("inclusive", "exclusive"):
+                    got = _run(x, op, kind, "cluster", 32 * variant + csize)
+                    assert_parity(got, x, op, kind, label="cluster v%d c%d %s %s %s N=%d G=%d" % (
+                        variant, csize, op, dt, kind, N, G))
 
 
 @pytest.mark.parametrize("K", [1, 2, 5])
