@@ -20,7 +20,7 @@ from . import _lib
 from ._lib import ALGOS, KINDS, OPS, ScanError, check
 
 __all__ = ["scan", "scan_host", "shard_totals", "shard_scan", "workspace_bytes", "ScanError",
-           "DTYPES"]
+           "DTYPES", "plan", "autotune", "autotune_clear"]
 
 DTYPES = {torch.int32: 0, torch.uint32: 1, torch.float32: 2}
 _NP_DTYPES = {np.dtype(np.int32): 0, np.dtype(np.uint32): 1, np.dtype(np.float32): 2}
@@ -158,6 +158,29 @@ def plan(x: torch.Tensor, out: torch.Tensor | None = None) -> tuple[str, int]:
     check("scan_plan", _lib.lib.scan_plan(N, G, x.data_ptr(), (out if out is not None else x).data_ptr(),
                                           ctypes.byref(a), ctypes.byref(pr)))
     return ALGO_NAMES[a.value], pr.value
+
+
+def autotune(x: torch.Tensor, op: str = "add", kind: str = "inclusive", out: torch.Tensor | None = None,
+             stream=None) -> tuple[str, int, float]:
+    """Time every kernel family / parameter that takes this shape on x -> out (out is
+    overwritten, must not be x) and make the fastest the AUTO choice for (N, G, alignment)
+    in this process (scan_autotune, the automated form of the paper's K search,
+    PAPER.md:183).  Synchronous.  Returns (algo, param, microseconds per call)."""
+    if out is None:
+        out = torch.empty_like(x)
+    _require_cuda(x, out)
+    N, G = _shape(x)
+    a, pr, us = ctypes.c_int(0), ctypes.c_int64(0), ctypes.c_float(0.0)
+    with torch.cuda.device(x.device):
+        rc = _lib.lib.scan_autotune(x.data_ptr(), out.data_ptr(), N, G, OPS[op], _dtype(x), KINDS[kind],
+                                    _stream(x, stream), ctypes.byref(a), ctypes.byref(pr), ctypes.byref(us))
+    check("scan_autotune", rc)
+    return ALGO_NAMES[a.value], pr.value, us.value
+
+
+def autotune_clear() -> None:
+    """Forget every tuned choice (AUTO falls back to the static dispatch rules)."""
+    check("scan_autotune_clear", _lib.lib.scan_autotune_clear())
 
 
 def abi_version() -> int:

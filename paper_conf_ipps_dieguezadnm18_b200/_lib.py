@@ -24,7 +24,8 @@ EXPORTS = ("scan_status_string", "scan_abi_version", "scan_batch", "scan_workspa
            "scan_batch_ex", "scan_batch_host", "scan_shard_totals", "scan_shard_scan",
            "scan_shard_workspace_bytes", "scan_debug_trace", "scan_plan", "scan_comm_create_nccl",
            "scan_comm_get_unique_id", "scan_comm_init_rank", "scan_comm_destroy", "scan_batch_multi",
-           "scan_comm_create_peer", "scan_comm_peer_handle", "scan_comm_peer_open")
+           "scan_comm_create_peer", "scan_comm_peer_handle", "scan_comm_peer_open", "scan_autotune",
+           "scan_autotune_clear")
 PEER_HANDLE_BYTES = 128
 SHARD = {"problems": 0, "elements": 1}
 
@@ -61,6 +62,8 @@ def _load() -> ctypes.CDLL:
         "scan_comm_create_peer": ([I, I, I64, P], I),
         "scan_comm_peer_handle": ([P, P], I),
         "scan_comm_peer_open": ([P, P], I),
+        "scan_autotune": ([P, P, I64, I64, I, I, I, P, P, P, P], I),
+        "scan_autotune_clear": ([], I),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -73,7 +76,7 @@ lib = _load()
 
 
 def lib_num_lookback_variants() -> int:
-    return 13
+    return 15
 
 
 def check(fn: str, code: int) -> None:

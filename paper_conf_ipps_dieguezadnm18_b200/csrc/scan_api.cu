@@ -23,6 +23,7 @@ namespace {
 constexpr size_t kCtlBytes = 256;          // [0] ticket [1] done [2] epoch (look-back)
 constexpr int kTargetCtas = 148 * 8;       // chunk count target of the three-stage path
 constexpr int64_t kMaxChunkTiles = 16;     // longest three-stage chunk (tiles of 4096)
+constexpr int64_t kFuse2MaxChunks = 256;   // Stage 2 folded into Stage 3 up to this many chunks
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
@@ -69,7 +70,12 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // cluster per problem (DSMEM aggregates) up to 2^15 (2^16 for G <= 4): ~3.7-4.6 us
     if (G <= 148 && N <= 8192) return SCAN_ALGO_CASCADE_CTA;
     if ((G <= 64 && N <= 32768) || (G <= 4 && N <= 65536)) return SCAN_ALGO_CLUSTER;
-    if (G <= 16 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    if (G <= 64 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    // a few hundred to a few thousand problems of moderate length (scan_autotune over a
+    // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA
+    // beat the flat look-back 1.1-4.8x there (e.g. G = 1024, N = 4096: 5.9 us vs 28 us)
+    if (G > 148 && N <= 1024 && N * G <= (int64_t(1) << 20)) return SCAN_ALGO_CASCADE_WARP;
+    if (G > 148 && N > 1024 && N <= 65536) return SCAN_ALGO_CASCADE_CTA;
     // short rows: several whole problems per warp (power-of-two N <= 512 flag-free)
     if (aligned && N < 1024) return SCAN_ALGO_PACKED_WARP;
     return SCAN_ALGO_LOOKBACK;
@@ -267,6 +273,15 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
     p.carry_src = carry_src;
     p.carry_rows = carry_rows;
     const OpCode oc = opcode(op, dt);
+    if (stages12 && stage3 && !totals_out && !peer && p.Bx <= kFuse2MaxChunks) {
+        // few chunks per problem and nobody needs the totals: Stage 2 is folded into
+        // Stage 3's prologue (two launches instead of three; latency-bound totals)
+        cudaError_t e = launch_chunk_reduce(oc, p, s);
+        if (e != cudaSuccess) return SCAN_ERR_CUDA;
+        p.aux_raw = true;
+        p.pdl = true;                                        // Stage 3 overlaps Stage 1's tail
+        return from_cuda(launch_chunk_scan(oc, p, s));
+    }
     if (stages12) {
         cudaError_t e = launch_chunk_reduce(oc, p, s);       // normal launch: waits for the caller's work
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
@@ -281,15 +296,37 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
     return SCAN_OK;
 }
 
+// ---------------------------------------------------------------- tuned choices
+// Filled by scan_autotune (the automated form of the paper's empirical K search,
+// PAPER.md:183): exact shape (N, G, base-pointer alignment) -> measured fastest family
+// and parameter.  SCAN_ALGO_AUTO consults it before the static rules.
+using TuneKey = std::tuple<int64_t, int64_t, bool>;
+std::mutex g_tune_mu;
+std::map<TuneKey, std::pair<scan_algo, int64_t>> g_tuned;
+
+bool tuned_choice(int64_t N, int64_t G, bool aligned, scan_algo* algo, int64_t* param) {
+    std::lock_guard<std::mutex> lk(g_tune_mu);
+    auto it = g_tuned.find(TuneKey(N, G, aligned));
+    if (it == g_tuned.end()) return false;
+    *algo = it->second.first;
+    *param = it->second.second;
+    return true;
+}
+
 scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dt,
                      scan_kind kind, scan_algo algo, int64_t param, void* ws, size_t ws_bytes,
                      cudaStream_t s) {
     if (algo == SCAN_ALGO_AUTO) {
-        algo = choose_algo(N, G, (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0));
-        // a caller workspace is sized and laid out for the look-back family
-        // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage scratch into it
-        if (ws && algo == SCAN_ALGO_THREE_STAGE) algo = SCAN_ALGO_LOOKBACK;
-        param = -1;
+        const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+        // a caller workspace is sized for the static choice (scan_workspace_bytes(AUTO)),
+        // so tuned choices apply only with the library's own workspace
+        if (ws || !tuned_choice(N, G, aligned, &algo, &param)) {
+            algo = choose_algo(N, G, aligned);
+            // a caller workspace is sized and laid out for the look-back family
+            // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage scratch into it
+            if (ws && algo == SCAN_ALGO_THREE_STAGE) algo = SCAN_ALGO_LOOKBACK;
+            param = -1;
+        }
     }
     switch (algo) {
     case SCAN_ALGO_LOOKBACK: {
@@ -484,6 +521,13 @@ scan_status scan_debug_trace(void* device_buf, int64_t tiles) {
 scan_status scan_plan(int64_t N, int64_t G, const void* in, const void* out, int* algo, int64_t* param) {
     if (!algo || !param || N < 0 || G < 0) return SCAN_ERR_INVALID_ARG;
     const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+    scan_algo ta;
+    int64_t tp;
+    if (tuned_choice(N, G, aligned, &ta, &tp)) {
+        *algo = (int)ta;
+        *param = tp;
+        return SCAN_OK;
+    }
     const scan_algo a = choose_algo(N, G, aligned);
     *algo = (int)a;
     *param = a == SCAN_ALGO_LOOKBACK ? choose_lookback_variant(N, G) : -1;
@@ -524,6 +568,111 @@ scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_
 scan_status scan_batch(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
                        scan_kind kind, void* stream) {
     return scan_batch_ex(in, out, N, G, op, dtype, kind, SCAN_ALGO_AUTO, -1, nullptr, 0, stream);
+}
+
+scan_status scan_autotune(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
+                          scan_kind kind, void* stream, int* algo_out, int64_t* param_out, float* us_out) {
+    if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
+    int64_t total = 0;
+    scan_status st = check_shape(N, G, &total);
+    if (st != SCAN_OK) return st;
+    if (total == 0) return SCAN_ERR_INVALID_ARG;
+    st = check_buffers(in, out, total, true);
+    if (st != SCAN_OK) return st;
+    if (in == out) return SCAN_ERR_INVALID_ARG;          // timing runs would rescan the output
+    cudaStream_t s = (cudaStream_t)stream;
+    const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+    // candidates: every family that takes this shape at a sane cost (a single CTA or warp
+    // per problem is excluded for few long problems: it would run for seconds)
+    std::vector<std::pair<scan_algo, int64_t>> cand;
+    for (int v : {0, 1, 2, 3, 10}) cand.push_back({SCAN_ALGO_LOOKBACK, v});
+    for (int k : {0, 1, 2, 4}) cand.push_back({SCAN_ALGO_THREE_STAGE, k});
+    if (G >= 64 || N <= (int64_t(1) << 16)) cand.push_back({SCAN_ALGO_CASCADE_CTA, -1});
+    if (G >= 256 && N <= (int64_t(1) << 16)) cand.push_back({SCAN_ALGO_CASCADE_WARP, -1});
+    if (aligned && N < 1024) cand.push_back({SCAN_ALGO_PACKED_WARP, -1});
+    if (N <= (int64_t(1) << 20) && G * kMaxClusterCtas <= 0x7FFFFFFFll)
+        for (int v = 0; v < 3; ++v)
+            for (int c : {2, 4, 8, 16}) cand.push_back({SCAN_ALGO_CLUSTER, 32 * v + c});
+    // Device time per call, measured like the on-box sweeps: `reps` calls captured into a
+    // CUDA graph on the library's tuning stream and replayed between two events, so host
+    // launch overhead does not pick the winner of small, latency-bound shapes.
+    cudaStream_t ts = nullptr;
+    {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess) return SCAN_ERR_NO_DEVICE;
+        static std::map<int, cudaStream_t> streams;          // one per device, kept (its
+        std::lock_guard<std::mutex> lk(g_tune_mu);            // workspaces are cached)
+        auto it = streams.find(dev);
+        if (it == streams.end()) {
+            if (cudaStreamCreateWithFlags(&ts, cudaStreamNonBlocking) != cudaSuccess) return SCAN_ERR_CUDA;
+            streams[dev] = ts;
+        } else {
+            ts = it->second;
+        }
+    }
+    if (cudaStreamSynchronize(s) != cudaSuccess) return SCAN_ERR_CUDA;     // the caller's inputs
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess) return SCAN_ERR_CUDA;
+    if (cudaEventCreate(&e1) != cudaSuccess) { cudaEventDestroy(e0); return SCAN_ERR_CUDA; }
+    float best = -1.0f;
+    std::pair<scan_algo, int64_t> win{SCAN_ALGO_AUTO, -1};
+    st = SCAN_OK;
+    for (const auto& c : cand) {
+        // warm-up call outside any capture (workspace growth, first-launch attributes); a
+        // family that rejects the shape is skipped
+        if (run_algo(in, out, N, G, op, dtype, kind, c.first, c.second, nullptr, 0, ts) != SCAN_OK ||
+            cudaStreamSynchronize(ts) != cudaSuccess) {
+            cudaGetLastError();
+            continue;
+        }
+        float ms1 = 0.0f;
+        if (cudaEventRecord(e0, ts) != cudaSuccess) { st = SCAN_ERR_CUDA; break; }
+        run_algo(in, out, N, G, op, dtype, kind, c.first, c.second, nullptr, 0, ts);
+        if (cudaEventRecord(e1, ts) != cudaSuccess || cudaEventSynchronize(e1) != cudaSuccess ||
+            cudaEventElapsedTime(&ms1, e0, e1) != cudaSuccess) { st = SCAN_ERR_CUDA; break; }
+        if (best > 0.0f && ms1 > 20.0f * best) continue;          // far off: not worth more reps
+        const int reps = (int)std::min(20.0f, std::max(2.0f, 1.0f / std::max(ms1, 1e-3f)));
+        cudaGraph_t graph = nullptr;
+        cudaGraphExec_t exec = nullptr;
+        if (cudaStreamBeginCapture(ts, cudaStreamCaptureModeThreadLocal) != cudaSuccess) { st = SCAN_ERR_CUDA; break; }
+        bool ok = true;
+        for (int r = 0; r < reps && ok; ++r)
+            ok = run_algo(in, out, N, G, op, dtype, kind, c.first, c.second, nullptr, 0, ts) == SCAN_OK;
+        if (cudaStreamEndCapture(ts, &graph) != cudaSuccess) ok = false;
+        if (ok && cudaGraphInstantiate(&exec, graph, 0) != cudaSuccess) ok = false;
+        float ms = 0.0f;
+        if (ok) ok = cudaGraphLaunch(exec, ts) == cudaSuccess && cudaEventRecord(e0, ts) == cudaSuccess &&
+                     cudaGraphLaunch(exec, ts) == cudaSuccess && cudaEventRecord(e1, ts) == cudaSuccess &&
+                     cudaEventSynchronize(e1) == cudaSuccess && cudaEventElapsedTime(&ms, e0, e1) == cudaSuccess;
+        if (exec) cudaGraphExecDestroy(exec);
+        if (graph) cudaGraphDestroy(graph);
+        if (!ok) {                     // not capturable / failed: this candidate is skipped
+            cudaGetLastError();
+            cudaStreamSynchronize(ts);
+            continue;
+        }
+        ms /= reps;
+        if (best < 0.0f || ms < best) { best = ms; win = c; }
+    }
+    cudaStreamSynchronize(ts);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (st != SCAN_OK) return st;
+    if (best < 0.0f) return SCAN_ERR_UNSUPPORTED;
+    {
+        std::lock_guard<std::mutex> lk(g_tune_mu);
+        g_tuned[TuneKey(N, G, aligned)] = win;
+    }
+    if (algo_out) *algo_out = (int)win.first;
+    if (param_out) *param_out = win.second;
+    if (us_out) *us_out = best * 1e3f;
+    return SCAN_OK;
+}
+
+scan_status scan_autotune_clear(void) {
+    std::lock_guard<std::mutex> lk(g_tune_mu);
+    g_tuned.clear();
+    return SCAN_OK;
 }
 
 scan_status scan_batch_host(const void* in_host, void* out_host, int64_t N, int64_t G, scan_op op,

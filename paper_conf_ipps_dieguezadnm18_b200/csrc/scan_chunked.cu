@@ -289,7 +289,16 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
         } else {
             for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
         }
-        if (p.aux) carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
+        if (p.aux && p.aux_raw) {
+            // Stage 2 folded into Stage 3 (few chunks per problem): each warp reduces the
+            // raw reductions of the chunks before this one itself -- one L2 round trip
+            // instead of a third launch
+            C pre = Op::cidentity();
+            for (int64_t k = lane; k < c; k += 32) pre = Op::capply(pre, slot_get<C>(p.aux[g * p.Bx + k]));
+            carry = Op::capply(carry, warp_reduce_carry<Op>(pre));
+        } else if (p.aux) {
+            carry = Op::capply(carry, slot_get<C>(p.aux[g * p.Bx + c]));
+        }
         return carry;
     };
     C carry = Op::cidentity();

@@ -76,6 +76,8 @@ struct ChunkParams {
     int64_t carry_stride;   // elements between carry rows (0 means G)
     bool vec;
     bool exclusive;
+    bool aux_raw;           // aux holds the RAW chunk reductions (Stage 2 skipped): every
+                            // Stage 3 CTA folds those of the chunks before it itself
     bool pdl;               // launch as a programmatic dependent of the previous kernel of
                             // this library call (Stage 2 after Stage 1, Stage 3 after Stage 2)
     PeerParams peer;        // fused exchange (peer.on) -- sharded path only

@@ -320,6 +320,44 @@ def test_packed_short_rows(param):
 def test_auto_short_rows_use_packed():
     x = torch.zeros((4096, 300), dtype=torch.int32, device="cuda")
     assert sb.plan(x)[0] == "packed_warp"
-    assert sb.plan(x[:, :1].contiguous().view(4096, 1))[0] == "packed_warp"
+    assert sb.plan(torch.zeros((1 << 21, 1), dtype=torch.int32, device="cuda"))[0] == "packed_warp"
     y = torch.zeros((4096, 1000), dtype=torch.int32, device="cuda")
     assert sb.plan(y)[0] == "cascade_warp"
+
+
+def test_auto_dispatch_regions():
+    # the measured regions of choose_algo (profiles/r01_cluster_probe.jsonl,
+    # r01_autotune_probe.jsonl); each shape must also scan exactly through AUTO
+    want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 65536): "cluster",
+            (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
+            (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 23): "lookback",
+            (4096, 16384): "cascade_cta"}
+    sb.autotune_clear()
+    for (G, N), algo in want.items():
+        x = inputs.generate("i32", G * N, seed=G + N).reshape(G, N)
+        xd = to_device(x)
+        assert sb.plan(xd)[0] == algo, (G, N, sb.plan(xd))
+        out = sb.scan(xd, "add", "exclusive")
+        torch.cuda.synchronize()
+        assert_parity(to_host(out, x.dtype), x, "add", "exclusive", label="auto G=%d N=%d" % (G, N))
+
+
+def test_autotune_table():
+    # scan_autotune (the automated K search of PAPER.md:183): the measured winner becomes
+    # the AUTO choice for that exact shape, results stay exact, clear() restores the rules
+    sb.autotune_clear()
+    for G, N in [(1, 20000), (3, 100003), (512, 1000)]:
+        x = inputs.generate("i32", G * N, seed=G + N).reshape(G, N)
+        xd = to_device(x)
+        before = sb.plan(xd)
+        algo, param, us = sb.autotune(xd, "add", "inclusive")
+        assert algo in sb.ALGOS and algo != "auto" and us > 0.0
+        assert sb.plan(xd) == (algo, param)
+        for op, dt in COMBOS:
+            xx = inputs.generate(DIST[dt], G * N, seed=3 * G + N).reshape(G, N)
+            for kind in ("inclusive", "exclusive"):
+                assert_parity(_run(xx, op, kind), xx, op, kind, label="tuned %s/%d %s %s" % (algo, param, op, dt))
+        sb.autotune_clear()
+        assert sb.plan(xd) == before
+    with pytest.raises(sb.ScanError):
+        sb.autotune(xd, "add", "inclusive", out=xd)          # in-place tuning is rejected
