@@ -254,7 +254,8 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
-    __shared__ T s_wval[2][WARPS];
+    static_assert(WARPS % 4 == 0, "warp slots are read as 16-byte vectors");
+    __shared__ __align__(16) T s_wval[2][WARPS];
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t g = (int64_t)blockIdx.x / p.Bx, c = (int64_t)blockIdx.x % p.Bx;
     const int64_t row = g * p.N;
@@ -310,12 +311,24 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
         wt.scan();
         if (lane == 0) s_wval[it & 1][warp] = wt.wtot;
         __syncthreads();
+        // the WARPS slots of this tile's buffer, read as exactly WARPS/4 16-byte vectors
+        // (double-buffered by tile parity: one barrier per tile; slot it&1 is rewritten in
+        // tile it+2, after barrier it+1, which every warp reaches after these reads)
+        T wv[WARPS];
+#pragma unroll
+        for (int q = 0; q < WARPS / 4; ++q) {
+            uint4 u;
+            asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(u.x), "=r"(u.y), "=r"(u.z), "=r"(u.w)
+                         : "r"(smem_u32(&s_wval[it & 1][4 * q])) : "memory");
+            wv[4 * q] = from_bits<T>(u.x); wv[4 * q + 1] = from_bits<T>(u.y);
+            wv[4 * q + 2] = from_bits<T>(u.z); wv[4 * q + 3] = from_bits<T>(u.w);
+        }
         T wp = Op::identity(), tot = Op::identity();
 #pragma unroll
         for (int w = 0; w < WARPS; ++w) {
-            T v = s_wval[it & 1][w];
-            if (w < warp) wp = Op::apply(wp, v);
-            tot = Op::apply(tot, v);
+            if (w < warp) wp = Op::apply(wp, wv[w]);
+            tot = Op::apply(tot, wv[w]);
         }
         wt.store(out, wb, row + end, p.vec, wp, false, Op::from_carry(carry), p.exclusive);
         carry = Op::capply(carry, Op::to_carry(tot));
