@@ -42,23 +42,25 @@ OpCode opcode(scan_op op, scan_dtype dt) {
 
 bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == SCAN_F32; }
 
-// ---------------------------------------------------------------- dispatch (DESIGN.md §6)
-// The analogue of the paper's empirical K search: the thresholds below come
-// from the on-box sweep recorded in profiles/ (bench.py --sweep).
+// ---------------------------------------------------------------- dispatch (DESIGN.md §5)
+// The analogue of the paper's empirical K search: the regions below come
+// from on-box sweeps recorded in profiles/ (bench.py --sweep, tools/*_probe.py, and the
+// scan_autotune grid r01_autotune_probe.jsonl); scan_autotune overrides them per shape.
 //   many problems of moderate N (rows 16-byte aligned): the paper's own batch mapping wins
 //     on B200 -- one CTA per problem (cascade, L_y = 1) for N >= 4096, one warp per problem
 //     (L_y = 8) for 768 <= N < 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
-//   short rows (N < 1024, 16-byte aligned base pointers): several whole problems per warp
-//     (packed_warp; power-of-two N <= 512 at ~104 % of copy, ragged N ~85-91 %), against
-//     ~65-78 % for the flat segmented look-back (tools/short_probe.py);
-//   small totals of few problems (<= 2^22 elements, L2 resident, latency bound): the
-//     paper's three-stage form -- three short kernels beat one persistent look-back launch
-//     in device time (configs[0]: ~5 us vs ~7.5 us);
+//   few short / medium problems (latency bound): one CTA per problem (G <= 148, N <= 8192),
+//     one thread-block cluster per problem (N <= 2^15, 2^16 for G <= 4), then the paper's
+//     three-stage form (G <= 64, G*N <= 2^23; two launches while <= 256 chunks);
+//   a few hundred to a few thousand problems up to 2^16: CTA / warp per problem again
+//     (1.1-4.8x over the flat look-back);
+//   short rows (N < 1024, 16-byte aligned base pointers, large totals): several whole
+//     problems per warp (packed_warp; power-of-two N <= 512 at ~104 % of copy);
 //   everything else (few large problems, unaligned pointers): single-pass look-back
 //     (L2-staged variant for G*N >= 2^22, one-tile-per-CTA for short unaligned rows).
 //   (boundary re-measured with 64-byte descriptor slots, profiles/r01_boundary.txt: the
-//    look-back matches or beats the CTA cascade up to G = 2048; the cascade wins from
-//    G = 4096, where every SM holds many whole problems)
+//    look-back matches or beats the CTA cascade up to G = 2048 for N >= 2^17; the cascade
+//    wins from G = 4096, where every SM holds many whole problems)
 // `aligned` = both base pointers 16-byte aligned.
 scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
@@ -70,7 +72,10 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // cluster per problem (DSMEM aggregates) up to 2^15 (2^16 for G <= 4): ~3.7-4.6 us
     if (G <= 148 && N <= 8192) return SCAN_ALGO_CASCADE_CTA;
     if ((G <= 64 && N <= 32768) || (G <= 4 && N <= 65536)) return SCAN_ALGO_CLUSTER;
-    if (G <= 64 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    // three-stage up to 2^23 elements: the second read of the input still hits L2, and
+    // the chain beats the L2-staged look-back's fill/drain there (2^23: 16.3 vs 19.6 us;
+    // from 2^24 the look-back wins, profiles/r01_mid_probe.jsonl)
+    if (G <= 64 && N * G <= (int64_t(1) << 23) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     // a few hundred to a few thousand problems of moderate length (scan_autotune over a
     // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA
     // beat the flat look-back 1.1-4.8x there (e.g. G = 1024, N = 4096: 5.9 us vs 28 us)
@@ -112,7 +117,13 @@ int64_t three_stage_chunk(int64_t N, int64_t G, int64_t K) {
     // against 5.6-5.7 us at K = 2), two tiles up to 2^22 (configs[0], 2^20: 5.5 us against
     // 5.7 us at K = 1); tools/g1_probe.py, profiles/r01_g1_probe.jsonl
     if (N * G <= (int64_t(1) << 19)) return tile;
-    if (N * G <= (int64_t(1) << 22)) return 2 * tile;
+    // up to 2^22: at least two tiles, and few enough chunks (<= kFuse2MaxChunks) that Stage
+    // 2 folds into Stage 3 (2^22: 10.3 us against 11.9 us as three launches,
+    // profiles/r01_mid_probe.jsonl)
+    if (N * G <= (int64_t(1) << 22)) {
+        const int64_t c = (N + kFuse2MaxChunks - 1) / kFuse2MaxChunks;
+        return std::max<int64_t>(2 * tile, (c + tile - 1) / tile * tile);
+    }
     int64_t bx = std::max<int64_t>(1, (kTargetCtas + G - 1) / G);
     int64_t chunk = (N + bx - 1) / bx;
     chunk = std::max<int64_t>(tile, (chunk + tile - 1) / tile * tile);

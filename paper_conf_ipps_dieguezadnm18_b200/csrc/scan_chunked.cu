@@ -55,7 +55,7 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
-    __shared__ C s_part[WARPS];
+    __shared__ __align__(16) C s_part[(WARPS + 3) & ~3];
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t g = (int64_t)blockIdx.x / p.Bx, c = (int64_t)blockIdx.x % p.Bx;
     const int64_t row = g * p.N;
@@ -169,7 +169,7 @@ __device__ __forceinline__ void aux_scan_problem(const ChunkParams& p, int64_t g
 template <class Op, int WARPS>
 __global__ void __launch_bounds__(WARPS * 32) aux_scan_cta_kernel(ChunkParams p) {
     using C = typename Op::Carry;
-    __shared__ C s_w[WARPS];
+    __shared__ __align__(16) C s_w[(WARPS + 3) & ~3];
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t g = blockIdx.x;
     const PeerParams& pp = p.peer;

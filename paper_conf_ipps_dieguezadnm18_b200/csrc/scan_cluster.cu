@@ -37,7 +37,7 @@ __global__ void __launch_bounds__(WARPS * 32) cluster_scan_kernel(ChunkParams p)
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
-    __shared__ T s_wval[WARPS];
+    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
     __shared__ C s_agg[2];
     cg::cluster_group cl = cg::this_cluster();
     const unsigned csize = cl.num_blocks(), crank = cl.block_rank();

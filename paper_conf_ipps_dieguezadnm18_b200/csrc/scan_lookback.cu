@@ -277,8 +277,8 @@ __global__ void __launch_bounds__((WARPS + 1) * 32) lookback_persistent_kernel(L
     __shared__ uint32_t s_seg[S], s_fast[S];
     __shared__ uint32_t s_tag;
     __shared__ C s_carry;
-    __shared__ T s_wval[WARPS];
-    __shared__ uint32_t s_wflag[WARPS];
+    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
+    __shared__ __align__(16) uint32_t s_wflag[(WARPS + 3) & ~3];
     const int warp = threadIdx.x >> 5, lane = lane_id();
 
     if (threadIdx.x == 0) {
@@ -1056,8 +1056,8 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
     __shared__ int64_t s_tile_id, s_r;
     __shared__ uint32_t s_tag, s_seg, s_fast;
     __shared__ C s_carry;
-    __shared__ T s_wval[WARPS];
-    __shared__ uint32_t s_wflag[WARPS];
+    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
+    __shared__ __align__(16) uint32_t s_wflag[(WARPS + 3) & ~3];
     const int warp = threadIdx.x >> 5, lane = lane_id();
 
     // tiles follow blockIdx (blocks are dispatched in index order, so every tile a CTA
@@ -1158,8 +1158,8 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackPa
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4;
-    __shared__ T s_wval[WARPS];
-    __shared__ uint32_t s_wflag[WARPS];
+    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
+    __shared__ __align__(16) uint32_t s_wflag[(WARPS + 3) & ~3];
     __shared__ C s_carry;
     const int64_t tile = blockIdx.x;
     const TileInfo ti = classify(p, tile, TILE);
@@ -1183,7 +1183,7 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_cluster_kernel(LookbackPa
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
-    __shared__ T s_wval[WARPS];
+    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
     __shared__ C s_agg, s_carry;
     cg::cluster_group cl = cg::this_cluster();
     const unsigned crank = cl.block_rank();
