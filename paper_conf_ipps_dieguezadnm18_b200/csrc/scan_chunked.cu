@@ -65,16 +65,24 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     grid_dep_launch();          // Stage 2 may be scheduled now; it waits for our results
 
     C acc = Op::cidentity();
-    for (int64_t off = start + warp * WCH; off < end; off += TILE) {
-        Row4<T> x[V];
+    // two tiles per iteration: both tiles' rows are in flight before either is reduced
+    // (one memory latency per 2 tiles; rows past the chunk end load as the identity)
+    for (int64_t off = start + warp * WCH; off < end; off += 2 * TILE) {
+        Row4<T> x[2 * V];
 #pragma unroll
         for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, row + off + j * 128 + lane * 4, row + end, p.vec);
-        T t = Op::identity();
 #pragma unroll
         for (int j = 0; j < V; ++j)
+            x[V + j] = load_row<Op>(in, row + off + TILE + j * 128 + lane * 4, row + end, p.vec);
 #pragma unroll
-            for (int k = 0; k < 4; ++k) t = Op::apply(t, x[j].v[k]);
-        acc = Op::capply(acc, Op::to_carry(t));
+        for (int h = 0; h < 2; ++h) {
+            T t = Op::identity();
+#pragma unroll
+            for (int j = 0; j < V; ++j)
+#pragma unroll
+                for (int k = 0; k < 4; ++k) t = Op::apply(t, x[h * V + j].v[k]);
+            acc = Op::capply(acc, Op::to_carry(t));
+        }
     }
     acc = warp_reduce_carry<Op>(acc);
     if (lane == 0) s_part[warp] = acc;
