@@ -1,0 +1,123 @@
+"""Perf-regression floors on the BASELINE configs, read from
+tests/perf_floors.json.  The floors sit well below the measured round-1 numbers
+(profiles/r01_bench_n1.json, r01_paper_sweep_*.jsonl): they catch a dispatch mistake or a
+kernel regression, not box-to-box noise.  Device time from CUDA events (large configs) or
+CUDA-graph replays (latency-bound ones)."""
+import json
+import os
+
+import pytest
+import torch
+
+import inputs
+import paper_conf_ipps_dieguezadnm18_b200 as sb
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+FLOORS = json.load(open(os.path.join(os.path.dirname(__file__), "perf_floors.json")))
+
+
+def _peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    return float(json.load(open(p))["hbm_gbs"]) if os.path.exists(p) else 6650.0
+
+
+def _ms(fn, reps):
+    for _ in range(2):
+        fn()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    s0.record()
+    for _ in range(reps):
+        fn()
+    s1.record()
+    torch.cuda.synchronize()
+    return s0.elapsed_time(s1) / reps
+
+
+def _graph_us(fn, reps=20):
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            fn()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(reps):
+            fn()
+    g.replay()
+    torch.cuda.synchronize()
+    best = None
+    for _ in range(3):
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(s)
+        with torch.cuda.stream(s):
+            g.replay()
+        s1.record(s)
+        torch.cuda.synchronize()
+        t = s0.elapsed_time(s1) / reps * 1e3
+        best = t if best is None else min(best, t)
+    return best
+
+
+def _frac(elems, ms):
+    return 8.0 * elems / (ms * 1e-3) / 1e9 / _peak()
+
+
+def test_c2_batch_rate():
+    G, N = 4096, 1 << 14
+    for dist, dt in (("i32", torch.int32), ("f32u", torch.float32)):
+        x = torch.empty(G * N, dtype=torch.int32, device="cuda")
+        inputs.fill_device(x, dist, 2)
+        x = x.view(dt).view(G, N)
+        y = torch.empty_like(x)
+        for kind in ("inclusive", "exclusive"):
+            f = _frac(G * N, _ms(lambda: sb.scan(x, "add", kind, out=y), 20))
+            assert f >= FLOORS["c2_frac_min"], (dist, kind, f)
+
+
+def test_c3_single_problem_rate():
+    N = 1 << 30
+    x = torch.empty(N, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "f32u", 3)
+    x = x.view(torch.float32)
+    y = torch.empty_like(x)
+    f = _frac(N, _ms(lambda: sb.scan(x, "add", out=y), 5))
+    assert f >= FLOORS["c3_frac_min"], f
+
+
+def test_c4_rank_shard_rate():
+    # configs[3] per GPU at W = 8: 2^13 problems of 2^16
+    G, N = 1 << 13, 1 << 16
+    x = torch.empty(G * N, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 4)
+    x = x.view(G, N)
+    y = torch.empty_like(x)
+    f = _frac(G * N, _ms(lambda: sb.scan(x, "add", out=y), 10))
+    assert f >= FLOORS["c4_shard_frac_min"], f
+
+
+def test_paper_sweep_rates():
+    # the paper's workload: 2^28 int32 as G = 2^28/N problems
+    T = 1 << 28
+    x = torch.empty(T, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 5)
+    y = torch.empty_like(x)
+    for n in (10, 13, 16, 20, 24, 28):
+        N = 1 << n
+        xv, yv = x.view(T // N, N), y.view(T // N, N)
+        f = _frac(T, _ms(lambda: sb.scan(xv, "add", out=yv), 5))
+        assert f >= FLOORS["paper_sweep_frac_min"], (n, sb.plan(xv, yv), f)
+
+
+def test_latency_bound_configs():
+    x = torch.empty(1 << 20, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 1)
+    y = torch.empty_like(x)
+    us = _graph_us(lambda: sb.scan(x, "add", out=y))
+    assert us <= FLOORS["c1_us_max"], us                       # configs[0]
+    for N in (1 << 12, 1 << 15):                                # one CTA / one cluster
+        xv, yv = x[:N], y[:N]
+        us = _graph_us(lambda: sb.scan(xv, "add", out=yv))
+        assert us <= FLOORS["g1_small_us_max"], (N, sb.plan(xv, yv), us)
