@@ -213,6 +213,10 @@ scan_status resolve_ws(void* ws, size_t ws_bytes, size_t need, cudaStream_t s, i
     return cached_workspace(s, fam, need, out, out_bytes);
 }
 
+// cross-call programmatic dependent launch of the CTA cascade (SCANB200_NO_PDL=1 disables
+// it, for A/B measurements)
+const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
+
 // debug timeline buffer for the look-back kernels (scan_debug_trace)
 uint64_t* g_trace = nullptr;
 int64_t g_trace_tiles = 0;
@@ -352,6 +356,10 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
     case SCAN_ALGO_CASCADE_CTA: {
         ChunkParams p = chunk_params(in, out, N, G, kind);
         p.chunk = std::max<int64_t>(N, 1); p.Bx = 1;
+        // programmatic launch behind the stream's previous kernel: the CTAs are scheduled
+        // into the SMs its last wave frees and wait there (griddepcontrol.wait) before
+        // their first access, so back-to-back calls lose no launch gap
+        p.pdl = p.pdl_first = g_cross_pdl;
         return from_cuda(launch_chunk_scan(opcode(op, dt), p, s));
     }
     case SCAN_ALGO_CASCADE_WARP: {

@@ -271,6 +271,10 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
     const T* in = (const T*)p.in;
     T* out = (T*)p.out;
+    // the next kernel on the stream may be scheduled once every CTA of this grid has
+    // started (it waits for this grid's completion before touching memory)
+    grid_dep_launch();
+    if (p.pdl_first) grid_dep_wait();      // a previous call may still be writing our input
 
     // Stage 2 results folded in: carries of earlier ranks (sharded mode),
     // then the exclusive prefix of the chunks before this one.  Read after

@@ -78,6 +78,9 @@ struct ChunkParams {
     bool exclusive;
     bool aux_raw;           // aux holds the RAW chunk reductions (Stage 2 skipped): every
                             // Stage 3 CTA folds those of the chunks before it itself
+    bool pdl_first;         // cross-call programmatic launch: the kernel may start while the
+                            // stream's previous kernel (any kernel) finishes, and waits for it
+                            // (griddepcontrol.wait) before its FIRST memory access
     bool pdl;               // launch as a programmatic dependent of the previous kernel of
                             // this library call (Stage 2 after Stage 1, Stage 3 after Stage 2)
     PeerParams peer;        // fused exchange (peer.on) -- sharded path only
