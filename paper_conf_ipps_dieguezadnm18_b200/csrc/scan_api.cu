@@ -47,8 +47,8 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 // from on-box sweeps recorded in profiles/ (bench.py --sweep, tools/*_probe.py, and the
 // scan_autotune grid r01_autotune_probe.jsonl); scan_autotune overrides them per shape.
 //   many problems of moderate N (rows 16-byte aligned): the paper's own batch mapping wins
-//     on B200 -- one CTA per problem (cascade, L_y = 1) for N >= 4096, one warp per problem
-//     (L_y = 8) for 768 <= N < 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
+//     on B200 -- one CTA per problem (cascade, L_y = 1) for N > 4096, one warp per problem
+//     (L_y = 8) for 768 <= N <= 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
 //   few short / medium problems (latency bound): one CTA per problem (G <= 148, N <= 8192),
 //     one thread-block cluster per problem (N <= 2^15, 2^16 for G <= 4), then the paper's
 //     three-stage form (G <= 64, G*N <= 2^23; two launches while <= 256 chunks);
@@ -64,8 +64,10 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 // `aligned` = both base pointers 16-byte aligned.
 scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     const bool rows_aligned = aligned && (N % 4 == 0);
-    if (rows_aligned && G >= 4096 && N >= 4096) return SCAN_ALGO_CASCADE_CTA;
-    if (rows_aligned && G >= 1184 && N >= 768 && N < 4096) return SCAN_ALGO_CASCADE_WARP;
+    // (N = 4096 exactly: one warp per problem 102 % vs one CTA 93 % of copy at G = 2^16,
+    //  tools/n12_probe.py)
+    if (rows_aligned && G >= 4096 && N > 4096) return SCAN_ALGO_CASCADE_CTA;
+    if (rows_aligned && G >= 1184 && N >= 768 && N <= 4096) return SCAN_ALGO_CASCADE_WARP;
     // few short / medium problems (latency bound, tools/cluster_probe.py on B200,
     // profiles/r01_cluster_probe.jsonl): one CTA per problem up to 8192 elements
     // (~2.5-3.3 us per call against 5-12 us for three-stage / look-back), one thread-block
@@ -290,8 +292,11 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
     const OpCode oc = opcode(op, dt);
     if (stages12 && stage3 && !totals_out && !peer && p.Bx <= kFuse2MaxChunks) {
         // few chunks per problem and nobody needs the totals: Stage 2 is folded into
-        // Stage 3's prologue (two launches instead of three; latency-bound totals)
+        // Stage 3's prologue (two launches instead of three; latency-bound totals).
+        // Stage 1 is itself a cross-call programmatic launch (waits before reading).
+        p.pdl = p.pdl_first = g_cross_pdl;
         cudaError_t e = launch_chunk_reduce(oc, p, s);
+        p.pdl_first = false;
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
         p.aux_raw = true;
         p.pdl = true;                                        // Stage 3 overlaps Stage 1's tail
@@ -365,6 +370,7 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
     case SCAN_ALGO_CASCADE_WARP: {
         ChunkParams p = chunk_params(in, out, N, G, kind);
         p.chunk = std::max<int64_t>(N, 1); p.Bx = 1;
+        p.pdl = p.pdl_first = g_cross_pdl;
         return from_cuda(launch_warp_cascade(opcode(op, dt), p, s));
     }
     case SCAN_ALGO_PACKED_WARP: {
@@ -372,6 +378,7 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         ChunkParams p = chunk_params(in, out, N, G, kind);
         p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
         p.chunk = packed_span_problems(N, param); p.Bx = 1;
+        p.pdl = p.pdl_first = g_cross_pdl;
         return from_cuda(launch_packed_warp(opcode(op, dt), p, s));
     }
     case SCAN_ALGO_CLUSTER: {

@@ -63,6 +63,7 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
     const T* in = (const T*)p.in;
     grid_dep_launch();          // Stage 2 may be scheduled now; it waits for our results
+    if (p.pdl_first) grid_dep_wait();      // cross-call programmatic launch (ChunkParams)
 
     C acc = Op::cidentity();
     // two tiles per iteration: both tiles' rows are in flight before either is reduced
@@ -371,6 +372,8 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
     constexpr int WCH = V * 128;
     const int warp = threadIdx.x >> 5;
     const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    grid_dep_launch();
+    if (p.pdl_first) grid_dep_wait();      // cross-call programmatic launch (ChunkParams)
     if (g >= p.G) return;
     const int64_t row = g * p.N;
     const T* in = (const T*)p.in;
@@ -402,6 +405,8 @@ __global__ void __launch_bounds__(WARPS * 32) packed_warp_kernel(ChunkParams p) 
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t k = p.chunk;                       // problems per span
     const int64_t g0 = ((int64_t)blockIdx.x * WARPS + warp) * k;
+    grid_dep_launch();
+    if (p.pdl_first) grid_dep_wait();
     if (g0 >= p.G) return;
     const int64_t base = g0 * p.N;
     const int64_t end = min(g0 + k, p.G) * p.N;
@@ -447,6 +452,8 @@ __global__ void __launch_bounds__(WARPS * 32) packed_pow2_kernel(ChunkParams p) 
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t base = ((int64_t)blockIdx.x * WARPS + warp) * WCH;
     const int64_t total = p.N * p.G;
+    grid_dep_launch();
+    if (p.pdl_first) grid_dep_wait();
     if (base >= total) return;
     const T* in = (const T*)p.in;
     T* out = (T*)p.out;
@@ -500,14 +507,6 @@ __global__ void peer_ack_kernel(PeerParams pp) {
     for (int r = 0; r < pp.rank; ++r) st_release_sys_u64(pp.push_ack[r], pp.epoch);
 }
 
-template <class Op>
-cudaError_t reduce_op(const ChunkParams& p, cudaStream_t s) {
-    int64_t blocks = p.G * p.Bx;
-    if (blocks == 0) return cudaSuccess;
-    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    chunk_reduce_kernel<Op, CH_WARPS, CH_V><<<(unsigned)blocks, CH_WARPS * 32, 0, s>>>(p);
-    return cudaGetLastError();
-}
 // launch, as a programmatic dependent of the stream's previous kernel when p.pdl
 template <class Kern>
 cudaError_t launch_maybe_pdl(Kern kern, unsigned blocks, unsigned threads, const ChunkParams& p, cudaStream_t s) {
@@ -526,6 +525,13 @@ cudaError_t launch_maybe_pdl(Kern kern, unsigned blocks, unsigned threads, const
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     return cudaLaunchKernelEx(&cfg, kern, p);
+}
+template <class Op>
+cudaError_t reduce_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = p.G * p.Bx;
+    if (blocks == 0) return cudaSuccess;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    return launch_maybe_pdl(chunk_reduce_kernel<Op, CH_WARPS, CH_V>, (unsigned)blocks, CH_WARPS * 32, p, s);
 }
 template <class Op>
 cudaError_t auxscan_op(const ChunkParams& p, cudaStream_t s) {
@@ -548,8 +554,8 @@ template <class Op>
 cudaError_t warp_op(const ChunkParams& p, cudaStream_t s) {
     int64_t blocks = (p.G + WC_WARPS - 1) / WC_WARPS;
     if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    warp_cascade_kernel<Op, WC_WARPS, WC_V><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
-    return cudaGetLastError();
+    if (blocks == 0) return cudaSuccess;
+    return launch_maybe_pdl(warp_cascade_kernel<Op, WC_WARPS, WC_V>, (unsigned)blocks, WC_WARPS * 32, p, s);
 }
 template <class Op>
 cudaError_t packed_op(const ChunkParams& p, cudaStream_t s) {
@@ -560,17 +566,15 @@ cudaError_t packed_op(const ChunkParams& p, cudaStream_t s) {
         const int64_t blocks = (windows + WC_WARPS - 1) / WC_WARPS;
         if (blocks == 0) return cudaSuccess;
         if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-        if (p.exclusive) packed_pow2_kernel<Op, WC_WARPS, WC_V, true><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
-        else packed_pow2_kernel<Op, WC_WARPS, WC_V, false><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
-        return cudaGetLastError();
+        return p.exclusive ? launch_maybe_pdl(packed_pow2_kernel<Op, WC_WARPS, WC_V, true>, (unsigned)blocks, WC_WARPS * 32, p, s)
+                           : launch_maybe_pdl(packed_pow2_kernel<Op, WC_WARPS, WC_V, false>, (unsigned)blocks, WC_WARPS * 32, p, s);
     }
     const int64_t spans = (p.G + p.chunk - 1) / p.chunk;
     const int64_t blocks = (spans + WC_WARPS - 1) / WC_WARPS;
     if (blocks == 0) return cudaSuccess;
     if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    if (p.exclusive) packed_warp_kernel<Op, WC_WARPS, WC_V, true><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
-    else packed_warp_kernel<Op, WC_WARPS, WC_V, false><<<(unsigned)blocks, WC_WARPS * 32, 0, s>>>(p);
-    return cudaGetLastError();
+    return p.exclusive ? launch_maybe_pdl(packed_warp_kernel<Op, WC_WARPS, WC_V, true>, (unsigned)blocks, WC_WARPS * 32, p, s)
+                       : launch_maybe_pdl(packed_warp_kernel<Op, WC_WARPS, WC_V, false>, (unsigned)blocks, WC_WARPS * 32, p, s);
 }
 
 #define SCANB200_DISPATCH(fn)                                          \
