@@ -386,6 +386,7 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         cluster_config(N, param, &variant, &csize);
         if ((int64_t)G * csize > 0x7FFFFFFFll) return SCAN_ERR_UNSUPPORTED;
         ChunkParams p = chunk_params(in, out, N, G, kind);
+        p.pdl_first = g_cross_pdl;
         return from_cuda(launch_cluster_scan(opcode(op, dt), p, variant, csize, s));
     }
     case SCAN_ALGO_THREE_STAGE: {

@@ -46,6 +46,8 @@ __global__ void __launch_bounds__(WARPS * 32) cluster_scan_kernel(ChunkParams p)
     const T* in = (const T*)p.in + g * p.N;
     T* out = (T*)p.out + g * p.N;
     const int64_t R = (int64_t)csize * TILE;
+    grid_dep_launch();                     // cross-call programmatic launch (ChunkParams)
+    if (p.pdl_first) grid_dep_wait();
 
     C run = Op::cidentity();
     int k = 0;
@@ -87,13 +89,15 @@ cudaError_t launch_t(const ChunkParams& p, int csize, cudaStream_t s) {
     cfg.blockDim = dim3(WARPS * 32, 1, 1);
     cfg.dynamicSmemBytes = 0;
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = (unsigned)csize;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = p.pdl_first ? 2 : 1;
     return cudaLaunchKernelEx(&cfg, kern, p);
 }
 
