@@ -413,6 +413,10 @@ __global__ void __launch_bounds__(WARPS * 32) packed_warp_kernel(ChunkParams p) 
     const T* in = (const T*)p.in;
     T* out = (T*)p.out;
     const uint32_t N32 = (uint32_t)p.N;
+    // position of this lane's row inside its problem, advanced by 128 mod N per row (one
+    // compare-subtract instead of a division per row)
+    const uint32_t step = 128u % N32;
+    uint32_t r = (uint32_t)(lane * 4) % N32;
     C carry = Op::cidentity();                       // segmented: value since the last head
     for (int64_t off = base; off < end; off += WCH) {
         Row4<T> x[V];                                // the whole window in flight at once
@@ -421,7 +425,9 @@ __global__ void __launch_bounds__(WARPS * 32) packed_warp_kernel(ChunkParams p) 
         // then row by row: only the running carry lives across rows (few registers)
 #pragma unroll
         for (int j = 0; j < V; ++j) {
-            const unsigned hd = row_heads_small((uint32_t)(off - base) + j * 128 + lane * 4, 0u, N32);
+            const unsigned hd = row_heads_from_r(r, N32);
+            r += step;
+            if (r >= N32) r -= N32;
             T v = row_reduce<Op, true>(x[j], hd);
             const unsigned hm = __ballot_sync(FULL, hd != 0u);
             T lin; bool lfl;

@@ -240,6 +240,17 @@ __device__ __forceinline__ unsigned row_heads_small(uint32_t o, uint32_t r_tile,
     }
     return m;
 }
+// The same from r = (row offset) mod N, maintained incrementally by the caller (no
+// division per row).
+__device__ __forceinline__ unsigned row_heads_from_r(uint32_t r, uint32_t N) {
+    uint32_t k = r ? N - r : 0u;
+    unsigned m = 0;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        if (k < 4u) { m |= 1u << k; k += N; }
+    }
+    return m;
+}
 __device__ __forceinline__ unsigned row_heads_big(int o, int first) {
     int d = first - o;
     return (d >= 0 && d < 4) ? (1u << d) : 0u;
