@@ -3,6 +3,7 @@
 // write of tile it+2 follows the barrier of tile it+1, which every warp reaches only after
 // its reads of tile it.  `compute-sanitizer --tool racecheck ./race_dbuf` tells whether the
 // checker flags the idiom itself on sm_100a.
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -lineinfo -O3 -o race_dbuf race_dbuf.cu
 #include <cstdio>
 #include <cuda_runtime.h>
 
