@@ -4,6 +4,7 @@
 // %globaltimer durations of the first read round and of the whole wait.
 // Modes: 0 = publish then read (concurrent writers); 1 = read slots already published by a
 // previous launch (pure read latency); 2 = one single relaxed load of own slot.
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o desc_latency desc_latency.cu
 #include <cstdio>
 #include <cstdint>
 #include <vector>
