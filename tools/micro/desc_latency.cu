@@ -3,7 +3,8 @@
 // reads slots [0, cta) (4 per lane) until every tag is current.  Reports per-CTA
 // %globaltimer durations of the first read round and of the whole wait.
 // Modes: 0 = publish then read (concurrent writers); 1 = read slots already published by a
-// previous launch (pure read latency); 2 = one single relaxed load of own slot.
+// previous launch (pure read latency); 2 = one single relaxed load of own slot; 4 = as 0
+// after every CTA first loads a 32 KiB tile of a 4 MiB buffer (a register-tile scan CTA).
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o desc_latency desc_latency.cu
 #include <cstdio>
 #include <cstdint>
@@ -16,13 +17,25 @@ __device__ __forceinline__ uint64_t ldr(const uint64_t* p) { uint64_t v; asm vol
 __device__ __forceinline__ void str(uint64_t* p, uint64_t v) { asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory"); }
 __device__ __forceinline__ uint64_t ldv(const uint64_t* p) { uint64_t v; asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v; }
 
-__global__ void k(uint64_t* slots, int stride_words, uint64_t tag, int mode, uint64_t* out) {
+__global__ void k(uint64_t* slots, int stride_words, uint64_t tag, int mode, uint64_t* out, const uint4* data) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int b = blockIdx.x;
+    __shared__ unsigned s_red;
+    if (mode == 4) {
+        // like a register-tile scan CTA: load a 32 KiB tile of a 4 MiB buffer first
+        unsigned acc = 0;
+        for (int i = threadIdx.x; i < 2048; i += blockDim.x) {
+            uint4 v = data[(size_t)b * 2048 + i];
+            acc += v.x + v.y + v.z + v.w;
+        }
+        if (threadIdx.x == 0) s_red = 0;
+        __syncthreads();
+        atomicAdd(&s_red, acc);
+    }
     __syncthreads();
     if (warp != 0) return;
     uint64_t t0 = gtime();
-    if (mode == 0 && lane == 0) str(slots + (size_t)b * stride_words, (tag << 32) | (uint64_t)b);
+    if ((mode == 0 || mode == 4) && lane == 0) str(slots + (size_t)b * stride_words, (tag << 32) | (uint64_t)(b + (mode == 4 ? s_red : 0u)));
     uint64_t t1 = gtime();
     int rounds = 0;
     uint64_t tfirst = 0;
@@ -48,22 +61,25 @@ __global__ void k(uint64_t* slots, int stride_words, uint64_t tag, int mode, uin
 
 int main() {
     uint64_t *slots, *out;
+    uint4* data;
+    cudaMalloc(&data, 128 * 2048 * 16);
+    cudaMemset(data, 1, 128 * 2048 * 16);
     cudaMalloc(&slots, 128 * 256 * 8);
     cudaMalloc(&out, 128 * 4 * 8);
     cudaMemset(slots, 0, 128 * 256 * 8);
     for (int stride : {1, 2, 8, 16, 32}) {
-        for (int mode : {0, 1, 3}) {
+        for (int mode : {0, 1, 3, 4}) {
             for (int nthreads : {32, 512}) {
                 std::vector<double> first, total, rnd;
                 for (int rep = 0; rep < 20; ++rep) {
                     uint64_t tag = 1000 + rep + stride * 100 + mode * 10000 + nthreads;
-                    if (mode != 0) {
+                    if (mode != 0 && mode != 4) {
                         // pre-publish with this tag
                         std::vector<uint64_t> h(128 * stride, 0);
                         for (int i = 0; i < 128; ++i) h[(size_t)i * stride] = (tag << 32) | i;
                         cudaMemcpy(slots, h.data(), h.size() * 8, cudaMemcpyHostToDevice);
                     }
-                    k<<<128, nthreads>>>(slots, stride, tag, mode, out);
+                    k<<<128, nthreads>>>(slots, stride, tag, mode, out, data);
                     std::vector<uint64_t> o(128 * 4);
                     cudaMemcpy(o.data(), out, o.size() * 8, cudaMemcpyDeviceToHost);
                     if (rep < 5) continue;
