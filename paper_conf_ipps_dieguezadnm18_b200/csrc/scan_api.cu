@@ -579,6 +579,7 @@ size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, 
 scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
                           scan_kind kind, scan_algo algo, int64_t param, void* workspace,
                           size_t workspace_bytes, void* stream) {
+    NvtxRange nvtx_range("scan_batch");
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
     if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_CLUSTER) return SCAN_ERR_UNSUPPORTED;
     int64_t total = 0;
@@ -599,6 +600,7 @@ scan_status scan_batch(const void* in, void* out, int64_t N, int64_t G, scan_op 
 
 scan_status scan_autotune(const void* in, void* out, int64_t N, int64_t G, scan_op op, scan_dtype dtype,
                           scan_kind kind, void* stream, int* algo_out, int64_t* param_out, float* us_out) {
+    NvtxRange nvtx_range("scan_autotune");
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
     int64_t total = 0;
     scan_status st = check_shape(N, G, &total);
@@ -704,6 +706,7 @@ scan_status scan_autotune_clear(void) {
 
 scan_status scan_batch_host(const void* in_host, void* out_host, int64_t N, int64_t G, scan_op op,
                             scan_dtype dtype, scan_kind kind) {
+    NvtxRange nvtx_range("scan_batch_host");
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
     int64_t total = 0;
     scan_status st = check_shape(N, G, &total);
@@ -723,6 +726,7 @@ size_t scan_shard_workspace_bytes(int64_t N_local, int64_t G) {
 
 scan_status scan_shard_totals(const void* in_local, int64_t N_local, int64_t G, scan_op op, scan_dtype dtype,
                               void* totals_dev, void* workspace, size_t workspace_bytes, void* stream) {
+    NvtxRange nvtx_range("stage1+2 (chunk reduce, totals)");
     if (!valid_enums(op, dtype, SCAN_INCLUSIVE)) return SCAN_ERR_INVALID_ARG;
     int64_t total = 0;
     scan_status st = check_shape(N_local, G, &total);
@@ -745,6 +749,7 @@ scan_status scan_shard_totals(const void* in_local, int64_t N_local, int64_t G, 
 scan_status scan_shard_scan(const void* in_local, void* out_local, int64_t N_local, int64_t G, scan_op op,
                             scan_dtype dtype, scan_kind kind, const void* all_totals_dev, int rank, int ngpu,
                             void* workspace, size_t workspace_bytes, void* stream) {
+    NvtxRange nvtx_range("stage3 (scan + carry)");
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
     if (ngpu < 1 || rank < 0 || rank >= ngpu) return SCAN_ERR_INVALID_ARG;
     int64_t total = 0;

@@ -6,7 +6,18 @@
 
 #include "scan_b200.h"
 
+#include <nvtx3/nvToolsExt.h>
+
 namespace scanb200 {
+
+// NVTX range around a library call or phase (visible in Nsight Systems / Compute; a
+// no-op costing a few ns when no tool is attached).  Names mirror the paper's phases.
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 enum class OpCode : int { AddU32 = 0, MaxI32 = 1, MaxU32 = 2, MaxF32 = 3, AddF32 = 4 };
 

@@ -259,6 +259,7 @@ scan_status scan_comm_destroy(scan_comm_t c) {
 scan_status scan_batch_multi(const void* in_local, void* out_local, int64_t N_local, int64_t G, scan_op op,
                              scan_dtype dtype, scan_kind kind, void* stream, int ngpu, scan_comm_t comm,
                              scan_shard mode) {
+    scanb200::NvtxRange nvtx_range("scan_batch_multi");
     if (mode == SCAN_SHARD_PROBLEMS)          // Case 1: each rank scans its own problems
         return scan_batch(in_local, out_local, N_local, G, op, dtype, kind, stream);
     if (mode != SCAN_SHARD_ELEMENTS) return SCAN_ERR_UNSUPPORTED;
