@@ -363,6 +363,23 @@ def test_autotune_table():
         sb.autotune(xd, "add", "inclusive", out=xd)          # in-place tuning is rejected
 
 
+def test_autotune_with_caller_workspace():
+    # a caller workspace is sized for the static AUTO choice (scan_workspace_bytes(AUTO)):
+    # with one, AUTO must ignore the tuned table and still scan exactly
+    sb.autotune_clear()
+    G, N = 64, 65536                        # static rule: three-stage; with a workspace: look-back
+    x = inputs.generate("i32", G * N, seed=77).reshape(G, N)
+    xd = to_device(x)
+    sb.autotune(xd, "add", "inclusive")
+    nbytes = sb.workspace_bytes(N, G, "add", torch.int32, "auto")
+    ws = torch.zeros(nbytes, dtype=torch.uint8, device="cuda")
+    for kind in ("inclusive", "exclusive"):
+        out = sb.scan(xd, "add", kind, workspace=ws)
+        torch.cuda.synchronize()
+        assert_parity(to_host(out, np.int32), x, "add", kind, label="tuned + caller workspace")
+    sb.autotune_clear()
+
+
 @pytest.mark.parametrize("algo,G,N", [("cascade_cta", 512, 8192), ("cascade_warp", 2000, 1000),
                                       ("packed_warp", 20000, 100), ("cluster", 3, 30000),
                                       ("three_stage", 1, 1 << 20), ("auto", 4096, 4096)])
