@@ -50,7 +50,7 @@ bool split_desc(scan_op op, scan_dtype dt) { return op == SCAN_OP_ADD && dt == S
 //     on B200 -- one CTA per problem (cascade, L_y = 1) for N > 4096, one warp per problem
 //     (L_y = 8) for 768 <= N <= 4096: no inter-CTA traffic at all, ~6.3-6.8 TB/s measured;
 //   few short / medium problems (latency bound): one CTA per problem (G <= 148, N <= 8192),
-//     one thread-block cluster per problem (N <= 2^15, 2^16 for G <= 4), then the paper's
+//     one thread-block cluster per problem (N <= 2^15), then the paper's
 //     three-stage form (G <= 64, G*N <= 2^23; two launches while <= 256 chunks);
 //   a few hundred to a few thousand problems up to 2^16: CTA / warp per problem again
 //     (1.1-4.8x over the flat look-back);
@@ -71,9 +71,11 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // few short / medium problems (latency bound, tools/cluster_probe.py on B200,
     // profiles/r01_cluster_probe.jsonl): one CTA per problem up to 8192 elements
     // (~2.5-3.3 us per call against 5-12 us for three-stage / look-back), one thread-block
-    // cluster per problem (DSMEM aggregates) up to 2^15 (2^16 for G <= 4): ~3.7-4.6 us
+    // cluster per problem (DSMEM aggregates) up to 2^15: ~3.3-3.9 us
     if (G <= 148 && N <= 8192) return SCAN_ALGO_CASCADE_CTA;
-    if ((G <= 64 && N <= 32768) || (G <= 4 && N <= 65536)) return SCAN_ALGO_CLUSTER;
+    // (2^15 < N <= 2^16 at G = 1: the two-launch chain 3.6 us vs the cluster 3.9-4.0 us once
+    //  both use programmatic launch, profiles/r01_g1_probe_cluster_boundary.jsonl)
+    if (G <= 64 && N <= 32768) return SCAN_ALGO_CLUSTER;
     // three-stage up to 2^23 elements: the second read of the input still hits L2, and
     // the chain beats the L2-staged look-back's fill/drain there (2^23: 16.3 vs 19.6 us;
     // from 2^24 the look-back wins, profiles/r01_mid_probe.jsonl)

@@ -328,7 +328,7 @@ def test_auto_short_rows_use_packed():
 def test_auto_dispatch_regions():
     # the measured regions of choose_algo (profiles/r01_cluster_probe.jsonl,
     # r01_autotune_probe.jsonl); each shape must also scan exactly through AUTO
-    want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 65536): "cluster",
+    want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 32768): "cluster", (4, 65536): "three_stage",
             (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
             (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 23): "three_stage", (1, 1 << 24): "lookback",
             (4096, 16384): "cascade_cta"}
