@@ -265,6 +265,7 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     p.trace_tiles = g_trace_tiles;
     p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
     p.exclusive = kind == SCAN_EXCLUSIVE;
+    p.pdl_first = g_cross_pdl;
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
 }
 

@@ -34,6 +34,9 @@ struct LookbackParams {
     int64_t trace_tiles;
     bool vec;           // in and out are 16-byte aligned
     bool exclusive;
+    bool pdl_first;     // cross-call programmatic launch (L2-staged kernel): CTAs may be
+                        // scheduled while the stream's previous kernel drains and execute
+                        // griddepcontrol.wait before their first global memory access
 };
 // u64 words per look-back descriptor slot.  A descriptor needs 1 (32-bit carries) or 2
 // (fp64 carries) words; one descriptor per 64-byte slot puts only two tiles on a 128-byte

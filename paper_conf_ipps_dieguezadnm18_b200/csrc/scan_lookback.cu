@@ -822,6 +822,11 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     __shared__ uint32_t s_tag;
     __shared__ int64_t s_end;
     const int warp = threadIdx.x >> 5, lane = lane_id();
+    // every CTA is resident before a dependent grid can launch (launch_dependents counts
+    // all of them), so the static round robin's inter-CTA waits cannot be starved of SMs;
+    // the wait orders the previous kernel's writes (our input, the epoch) before any access
+    grid_dep_launch();
+    if (p.pdl_first) grid_dep_wait();
 
     if (threadIdx.x == 0) {
         s_end = INT64_MAX;
@@ -1039,8 +1044,17 @@ cudaError_t launch_l2(const LookbackParams& p, cudaStream_t s) {
     if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
     int64_t grid = (int64_t)occ * num_sms();
     if (grid > tiles) grid = tiles;
-    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid, 1, 1);
+    cfg.blockDim = dim3(THREADS, 1, 1);
+    cfg.dynamicSmemBytes = SMEM;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = p.pdl_first ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kern, p, tiles);
 }
 
 // ---------------------------------------------------------------- one tile per CTA (comparison)
