@@ -382,19 +382,22 @@ def test_autotune_with_caller_workspace():
 
 @pytest.mark.parametrize("algo,G,N", [("cascade_cta", 512, 8192), ("cascade_warp", 2000, 1000),
                                       ("packed_warp", 20000, 100), ("cluster", 3, 30000),
-                                      ("three_stage", 1, 1 << 20), ("auto", 4096, 4096)])
+                                      ("three_stage", 1, 1 << 20), ("auto", 4096, 4096),
+                                      ("lookback/3", 1, 1 << 22), ("lookback/3", 3, 1000003)])
 def test_back_to_back_ordering(algo, G, N):
     # the single-kernel families and Stage 1 are launched as programmatic dependents of the
     # stream's previous kernel and wait before their first access: chains of dependent
     # calls and torch kernels on one stream, with no synchronisation, must stay ordered
+    # (the L2-staged look-back, "lookback/3", is a programmatic dependent too)
+    algo, param = (algo.split("/")[0], int(algo.split("/")[1])) if "/" in algo else (algo, -1)
     x = inputs.generate("small", G * N, seed=G + N).reshape(G, N)
     ref = x
     xd = to_device(x)
     for r in range(3):
         xd.add_(1)                                              # torch kernel writes the input
-        y = sb.scan(xd, "add", "inclusive", algo=algo)          # reads it right behind
-        sb.scan(y, "max", "inclusive", out=y, algo=algo)        # in place, right behind
-        xd = sb.scan(y, "add", "exclusive", algo=algo)          # next round's input
+        y = sb.scan(xd, "add", "inclusive", algo=algo, param=param)     # reads it right behind
+        sb.scan(y, "max", "inclusive", out=y, algo=algo, param=param)   # in place, right behind
+        xd = sb.scan(y, "add", "exclusive", algo=algo, param=param)     # next round's input
         ref = (ref.astype(np.int64) + 1).astype(np.int32)        # wraps like torch int32 add_
         ref = oracle.scan(oracle.scan(ref, "add", "inclusive"), "max", "inclusive")
         ref = oracle.scan(ref, "add", "exclusive")
