@@ -15,6 +15,9 @@ Parity status of each function (pins are in tests/test_oracle.py):
   scan(..., 'max', *)     pinned: numpy maximum.accumulate, monotonicity, idempotence.
   scan(..., 'add', f32)   pinned: exact rational (fractions) sums on small inputs within
                           N*2^-53*sum|x|, closed form for 1..N while exact in fp64.
+  sabs (|x| prefix)       pinned: numpy cumsum(|x|) per problem (G >= 3, reset at every
+                          problem start), exclusive = sum over k < i (element 0 is 0),
+                          one-shot and StreamAdd (tests/test_oracle.py, test_sabs_*).
   exclusive kind          pinned: excl[0] = identity, excl[i] = incl[i-1].
   totals()                pinned: equals the last element of the inclusive scan and a
                           brute-force sum.

@@ -246,3 +246,62 @@ def test_streaming_oracle_equals_one_shot(dist, kind):
         assert np.array_equal(np.concatenate([p[1] for p in parts]), sabs)
     else:
         assert np.array_equal(np.concatenate(parts), oracle.scan(x, "add", kind))
+
+
+# ------------------------------------------------------------------ the |x| prefix (tolerance basis)
+# north_star: |err_i| <= 1e-5 * sum_{k<=i} |x_k| (inclusive); reading R3 takes
+# k < i for exclusive, so exclusive element 0 has bound 0 and must be exact.  The bound
+# itself comes from the oracle's `sabs`, so it is pinned here against an independent
+# numpy cumsum of |x| in fp64 -- per problem (G >= 3, reset at every problem start), for
+# both kinds, one-shot and streamed.  A sum over k <= i in the exclusive form, or a
+# missing reset between problems, fails these.
+def _abs_prefix_np(x2d):
+    return np.cumsum(np.abs(x2d.astype(np.float64)), axis=1)
+
+
+@pytest.mark.parametrize("dist", ["f32u", "f32s"])
+def test_sabs_inclusive_per_problem(dist):
+    G, N = 5, 1237
+    x = inputs.generate(dist, G * N, 41).reshape(G, N)
+    x[:, 0] = np.float32(0.75)                 # nonzero first element in every problem
+    _, sabs = oracle.scan(x, "add", "inclusive", with_abs=True)
+    ref_abs = _abs_prefix_np(x)
+    assert np.allclose(sabs, ref_abs, rtol=1e-12, atol=0)
+    # reset per problem: row g starts at |x[g,0]|, not at the previous row's total
+    assert np.all(sabs[:, 0] == np.float64(0.75))
+    assert np.all(np.diff(sabs, axis=1) >= 0)
+
+
+@pytest.mark.parametrize("dist", ["f32u", "f32s"])
+def test_sabs_exclusive_is_shifted_and_starts_at_zero(dist):
+    G, N = 4, 999
+    x = inputs.generate(dist, G * N, 43).reshape(G, N)
+    x[:, 0] = np.float32(-2.5)
+    _, sabs_e = oracle.scan(x, "add", "exclusive", with_abs=True)
+    _, sabs_i = oracle.scan(x, "add", "inclusive", with_abs=True)
+    assert np.all(sabs_e[:, 0] == 0.0)                       # empty range 0..-1 (reading R2/R3)
+    assert np.array_equal(sabs_e[:, 1:], sabs_i[:, :-1])     # sum over k < i
+    ref_abs = _abs_prefix_np(x)
+    assert np.allclose(sabs_e[:, 1:], ref_abs[:, :-1], rtol=1e-12, atol=0)
+    # the exclusive bound is strictly below the inclusive one by |x_i| (never k <= i)
+    assert np.allclose(sabs_i - sabs_e, np.abs(x.astype(np.float64)), rtol=1e-9, atol=1e-12)
+
+
+@pytest.mark.parametrize("kind", ["inclusive", "exclusive"])
+def test_stream_sabs_against_numpy(kind):
+    x = inputs.generate("f32s", 30011, 47)
+    x[0] = np.float32(1.5)
+    s = oracle.StreamAdd(np.float32, kind)
+    ys, sa = zip(*[s.feed(x[a:b]) for a, b in [(0, 3), (3, 8195), (8195, 8195), (8195, 30011)]])
+    sa = np.concatenate(sa)
+    ys = np.concatenate(ys)
+    ref_abs = np.cumsum(np.abs(x.astype(np.float64)))
+    ref_val = np.cumsum(x.astype(np.float64))
+    if kind == "exclusive":
+        assert sa[0] == 0.0 and ys[0] == 0.0
+        assert np.allclose(sa[1:], ref_abs[:-1], rtol=1e-12, atol=0)
+        assert np.allclose(ys[1:], ref_val[:-1], rtol=0, atol=1e-9)
+    else:
+        assert sa[0] == 1.5
+        assert np.allclose(sa, ref_abs, rtol=1e-12, atol=0)
+        assert np.allclose(ys, ref_val, rtol=0, atol=1e-9)
