@@ -467,7 +467,7 @@ def sweep(sb, dev):
               ("i32", 4096, 1 << 14), ("f32", 4096, 1 << 14), ("i32", 1 << 16, 1 << 10),
               ("i32", 1 << 14, 1 << 12), ("i32", 256, 1 << 20), ("i32", 16, 1 << 24), ("i32", 1 << 18, 1 << 8),
               ("i32", 1 << 20, 1 << 6), ("i32", 1 << 13, 1 << 16)]
-    cands = [("lookback", v) for v in range(sb._lib.lib_num_lookback_variants())] + [
+    cands = [("lookback", v) for v in sb._lib.LOOKBACK_VARIANTS] + [
         ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0)]
     s = torch.cuda.Stream(dev)
     for dt, G, N in shapes:

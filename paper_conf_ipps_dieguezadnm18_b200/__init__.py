@@ -151,20 +151,23 @@ KERNEL_NAMES = {"lookback": "lookback_*_kernel (decoupled look-back)",
                 "cluster": "cluster_scan_kernel (one thread-block cluster per problem, DSMEM aggregates)"}
 
 
-def plan(x: torch.Tensor, out: torch.Tensor | None = None) -> tuple[str, int]:
-    """The (algo, param) that algo='auto' picks for this tensor (scan_plan)."""
+def plan(x: torch.Tensor, out: torch.Tensor | None = None, op: str = "add",
+         kind: str = "inclusive") -> tuple[str, int]:
+    """The (algo, param) that algo='auto' picks for this tensor, op and kind (scan_plan_ex)."""
     N, G = _shape(x)
     a, pr = ctypes.c_int(0), ctypes.c_int64(0)
-    check("scan_plan", _lib.lib.scan_plan(N, G, x.data_ptr(), (out if out is not None else x).data_ptr(),
-                                          ctypes.byref(a), ctypes.byref(pr)))
+    with torch.cuda.device(x.device):
+        check("scan_plan_ex", _lib.lib.scan_plan_ex(N, G, OPS[op], _dtype(x), KINDS[kind], x.data_ptr(),
+                                                    (out if out is not None else x).data_ptr(),
+                                                    ctypes.byref(a), ctypes.byref(pr)))
     return ALGO_NAMES[a.value], pr.value
 
 
 def autotune(x: torch.Tensor, op: str = "add", kind: str = "inclusive", out: torch.Tensor | None = None,
              stream=None) -> tuple[str, int, float]:
     """Time every kernel family / parameter that takes this shape on x -> out (out is
-    overwritten, must not be x) and make the fastest the AUTO choice for (N, G, alignment)
-    in this process (scan_autotune, the automated form of the paper's K search,
+    overwritten, must not be x) and make the fastest the AUTO choice for (device, N, G,
+    alignment, op, dtype, kind) in this process (scan_autotune, the automated form of the paper's K search,
     PAPER.md:183).  Synchronous.  Returns (algo, param, microseconds per call)."""
     if out is None:
         out = torch.empty_like(x)

@@ -22,7 +22,7 @@ STATUS = {0: "SCAN_OK", 1: "SCAN_ERR_INVALID_ARG", 2: "SCAN_ERR_UNSUPPORTED", 3:
 # every symbol include/scan_b200.h declares (checked by tests/test_abi.py)
 EXPORTS = ("scan_status_string", "scan_abi_version", "scan_batch", "scan_workspace_bytes",
            "scan_batch_ex", "scan_batch_host", "scan_shard_totals", "scan_shard_scan",
-           "scan_shard_workspace_bytes", "scan_debug_trace", "scan_plan", "scan_comm_create_nccl",
+           "scan_shard_workspace_bytes", "scan_debug_trace", "scan_plan", "scan_plan_ex", "scan_comm_create_nccl",
            "scan_comm_get_unique_id", "scan_comm_init_rank", "scan_comm_destroy", "scan_batch_multi",
            "scan_comm_create_peer", "scan_comm_peer_handle", "scan_comm_peer_open", "scan_autotune",
            "scan_autotune_clear")
@@ -54,6 +54,7 @@ def _load() -> ctypes.CDLL:
         "scan_shard_workspace_bytes": ([I64, I64], SZ),
         "scan_debug_trace": ([P, I64], I),
         "scan_plan": ([I64, I64, P, P, P, P], I),
+        "scan_plan_ex": ([I64, I64, I, I, I, P, P, P, P], I),
         "scan_comm_create_nccl": ([P, I, I, P], I),
         "scan_comm_get_unique_id": ([P], I),
         "scan_comm_init_rank": ([P, I, I, P], I),
@@ -75,8 +76,8 @@ def _load() -> ctypes.CDLL:
 lib = _load()
 
 
-def lib_num_lookback_variants() -> int:
-    return 15
+# look-back kernel variants of the library (scan_lookback.cu: lookback_variant_valid)
+LOOKBACK_VARIANTS = (0, 1, 2, 3, 10)
 
 
 def check(fn: str, code: int) -> None:

@@ -183,8 +183,10 @@ size_t three_stage_bytes(int64_t N, int64_t G, int64_t K) {
 struct Ws { void* ptr = nullptr; size_t bytes = 0; };
 std::mutex g_ws_mu;
 // one cache per (device, stream, family): the look-back descriptors must never share
-// bytes with another family's scratch values
-enum Family { FAM_LOOKBACK = 0, FAM_CHUNKED = 1 };
+// bytes with another family's scratch values, and the chunk prefixes that
+// scan_shard_totals leaves for scan_shard_scan (FAM_SHARD) must survive any scan_batch
+// call the caller issues on the same stream between the two steps
+enum Family { FAM_LOOKBACK = 0, FAM_CHUNKED = 1, FAM_SHARD = 2 };
 std::map<std::tuple<int, cudaStream_t, int>, Ws> g_ws;
 
 scan_status cached_workspace(cudaStream_t s, int fam, size_t need, void** out, size_t* out_bytes) {
@@ -321,15 +323,23 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
 
 // ---------------------------------------------------------------- tuned choices
 // Filled by scan_autotune (the automated form of the paper's empirical K search,
-// PAPER.md:183): exact shape (N, G, base-pointer alignment) -> measured fastest family
-// and parameter.  SCAN_ALGO_AUTO consults it before the static rules.
-using TuneKey = std::tuple<int64_t, int64_t, bool>;
+// PAPER.md:183): exact problem (device, N, G, base-pointer alignment, op, dtype, kind) ->
+// measured fastest family and parameter.  SCAN_ALGO_AUTO consults it before the static
+// rules.  op / dtype / kind are part of the key because the cost differs (fp64 carries of
+// f32 add, the exclusive form), and the device because a process may drive several GPUs.
+using TuneKey = std::tuple<int, int64_t, int64_t, bool, int, int, int>;
 std::mutex g_tune_mu;
 std::map<TuneKey, std::pair<scan_algo, int64_t>> g_tuned;
 
-bool tuned_choice(int64_t N, int64_t G, bool aligned, scan_algo* algo, int64_t* param) {
+TuneKey tune_key(int64_t N, int64_t G, bool aligned, scan_op op, scan_dtype dt, scan_kind kind) {
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
+    return TuneKey(dev, N, G, aligned, (int)op, (int)dt, (int)kind);
+}
+
+bool tuned_choice(const TuneKey& key, scan_algo* algo, int64_t* param) {
     std::lock_guard<std::mutex> lk(g_tune_mu);
-    auto it = g_tuned.find(TuneKey(N, G, aligned));
+    auto it = g_tuned.find(key);
     if (it == g_tuned.end()) return false;
     *algo = it->second.first;
     *param = it->second.second;
@@ -343,7 +353,7 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
         // a caller workspace is sized for the static choice (scan_workspace_bytes(AUTO)),
         // so tuned choices apply only with the library's own workspace
-        if (ws || !tuned_choice(N, G, aligned, &algo, &param)) {
+        if (ws || !tuned_choice(tune_key(N, G, aligned, op, dt, kind), &algo, &param)) {
             algo = choose_algo(N, G, aligned);
             // a caller workspace is sized and laid out for the look-back family
             // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage scratch into it
@@ -353,7 +363,8 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
     }
     switch (algo) {
     case SCAN_ALGO_LOOKBACK: {
-        int variant = (param >= 0 && param < lookback_num_variants()) ? (int)param : choose_lookback_variant(N, G);
+        if (param >= 0 && !lookback_variant_valid((int)param)) return SCAN_ERR_UNSUPPORTED;
+        int variant = param >= 0 ? (int)param : choose_lookback_variant(N, G);
         void* w = nullptr;
         size_t wb = 0;
         scan_status st = resolve_ws(ws, ws_bytes, lookback_bytes(N * G, variant, split_desc(op, dt)), s,
@@ -548,12 +559,13 @@ scan_status scan_debug_trace(void* device_buf, int64_t tiles) {
     return SCAN_OK;
 }
 
-scan_status scan_plan(int64_t N, int64_t G, const void* in, const void* out, int* algo, int64_t* param) {
-    if (!algo || !param || N < 0 || G < 0) return SCAN_ERR_INVALID_ARG;
+scan_status scan_plan_ex(int64_t N, int64_t G, scan_op op, scan_dtype dtype, scan_kind kind, const void* in,
+                         const void* out, int* algo, int64_t* param) {
+    if (!algo || !param || N < 0 || G < 0 || !valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
     const bool aligned = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
     scan_algo ta;
     int64_t tp;
-    if (tuned_choice(N, G, aligned, &ta, &tp)) {
+    if (tuned_choice(tune_key(N, G, aligned, op, dtype, kind), &ta, &tp)) {
         *algo = (int)ta;
         *param = tp;
         return SCAN_OK;
@@ -564,6 +576,10 @@ scan_status scan_plan(int64_t N, int64_t G, const void* in, const void* out, int
     return SCAN_OK;
 }
 
+scan_status scan_plan(int64_t N, int64_t G, const void* in, const void* out, int* algo, int64_t* param) {
+    return scan_plan_ex(N, G, SCAN_OP_ADD, SCAN_I32, SCAN_INCLUSIVE, in, out, algo, param);
+}
+
 size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, scan_algo algo, int64_t param) {
     if (N <= 0 || G <= 0) return kCtlBytes;
     if (algo == SCAN_ALGO_AUTO) {
@@ -572,7 +588,8 @@ size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, 
         return lookback_bytes(N * G, 1, split_desc(op, dtype));
     }
     if (algo == SCAN_ALGO_LOOKBACK) {
-        int variant = (param >= 0 && param < lookback_num_variants()) ? (int)param : choose_lookback_variant(N, G);
+        if (param >= 0 && !lookback_variant_valid((int)param)) return kCtlBytes;
+        int variant = param >= 0 ? (int)param : choose_lookback_variant(N, G);
         return lookback_bytes(N * G, variant, split_desc(op, dtype));
     }
     if (algo == SCAN_ALGO_THREE_STAGE) return three_stage_bytes(N, G, param);
@@ -693,7 +710,7 @@ scan_status scan_autotune(const void* in, void* out, int64_t N, int64_t G, scan_
     if (best < 0.0f) return SCAN_ERR_UNSUPPORTED;
     {
         std::lock_guard<std::mutex> lk(g_tune_mu);
-        g_tuned[TuneKey(N, G, aligned)] = win;
+        g_tuned[tune_key(N, G, aligned, op, dtype, kind)] = win;
     }
     if (algo_out) *algo_out = (int)win.first;
     if (param_out) *param_out = win.second;
@@ -743,7 +760,7 @@ scan_status scan_shard_totals(const void* in_local, int64_t N_local, int64_t G, 
     }
     void* w = nullptr;
     size_t wb = 0;
-    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_CHUNKED, &w, &wb);
+    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_SHARD, &w, &wb);
     if (st != SCAN_OK) return st;
     return run_three_stage(in_local, nullptr, N_local, G, op, dtype, SCAN_INCLUSIVE, 0, w, nullptr, 0, s,
                            true, false, (uint64_t*)totals_dev);
@@ -765,7 +782,7 @@ scan_status scan_shard_scan(const void* in_local, void* out_local, int64_t N_loc
     cudaStream_t s = (cudaStream_t)stream;
     void* w = nullptr;
     size_t wb = 0;
-    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_CHUNKED, &w, &wb);
+    st = resolve_ws(workspace, workspace_bytes, three_stage_bytes(N_local, G, 0), s, FAM_SHARD, &w, &wb);
     if (st != SCAN_OK) return st;
     return run_three_stage(in_local, out_local, N_local, G, op, dtype, kind, 0, w,
                            (const uint64_t*)all_totals_dev, rank, s, false, true, nullptr);

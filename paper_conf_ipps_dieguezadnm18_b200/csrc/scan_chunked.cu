@@ -62,8 +62,15 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     const int64_t start = c * p.chunk;
     const int64_t end = (start + p.chunk < p.N) ? start + p.chunk : p.N;
     const T* in = (const T*)p.in;
-    grid_dep_launch();          // Stage 2 may be scheduled now; it waits for our results
+    // Ordering rule of the library: a kernel may touch memory before its own
+    // griddepcontrol.wait only if its primary executed the wait BEFORE it triggered.  The
+    // fused Stage 3 (aux_raw) loads its first input tile before waiting, so when this
+    // Stage 1 is itself a cross-call programmatic dependent (pdl_first) it waits for the
+    // stream's previous kernel -- which may trigger at entry and still be writing our
+    // input -- before letting Stage 3 launch.  Otherwise Stage 1 was a normal launch and
+    // everything before it is complete: trigger at once.
     if (p.pdl_first) grid_dep_wait();      // cross-call programmatic launch (ChunkParams)
+    grid_dep_launch();          // Stage 2 / fused Stage 3 may be scheduled now
 
     C acc = Op::cidentity();
     // two tiles per iteration: both tiles' rows are in flight before either is reduced

@@ -78,12 +78,9 @@ __global__ void __launch_bounds__(WARPS * 32) cluster_scan_kernel(ChunkParams p)
 template <class Op, int WARPS, int V>
 cudaError_t launch_t(const ChunkParams& p, int csize, cudaStream_t s) {
     auto kern = cluster_scan_kernel<Op, WARPS, V>;
-    static bool init = false;
-    if (!init) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (e != cudaSuccess) return e;
-        init = true;
-    }
+    // non-portable cluster sizes (16 CTAs) opted in once per device (scan_launch.cu)
+    cudaError_t e = kernel_prepare((const void*)kern, WARPS * 32, 0, true, nullptr);
+    if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(p.G * csize), 1, 1);
     cfg.blockDim = dim3(WARPS * 32, 1, 1);

@@ -542,83 +542,6 @@ struct WarpTileS {
     }
 };
 
-// Register-resident variant: pass 1 reads the warp's rows from shared memory ONCE and keeps
-// the warp-local (segmented) inclusive or exclusive prefix of every element in registers
-// (V x 4 values + one head bit per element), so the shared-memory slot can be released
-// before the carry is known; `emit` later adds the tile-level prefix and stores.
-template <class Op, int V>
-struct WarpTileR {
-    using T = typename Op::T;
-    static_assert(V * 4 <= 32, "one head bit per element in a 32-bit mask");
-    Row4<T> y[V];
-    uint32_t fm;          // bit 4j+k: a head at or before element (j,k) inside this warp window
-    T wtot; bool wfl;
-
-    template <bool SEG, bool EXCL>
-    __device__ __forceinline__ void pass1(const T* srow, int o0, bool small, uint32_t r_tile, uint32_t N32,
-                                          int first) {
-        const int lane = lane_id();
-        fm = 0u;
-        T run = Op::identity(); bool f = false;      // prefix of the rows before row j
-#pragma unroll
-        for (int j = 0; j < V; ++j) {
-            Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
-            unsigned hd = 0u;
-            if (SEG) {
-                int o = o0 + j * 128 + lane * 4;
-                hd = small ? row_heads_small((uint32_t)o, r_tile, N32) : row_heads_big(o, first);
-            }
-            T v = row_reduce<Op, SEG>(x, hd);
-            unsigned hm = SEG ? __ballot_sync(FULL, hd != 0u) : 0u;
-            T lin; bool lf;
-            T incl = warp_seg_scan<Op, SEG>(v, hm, lin, lf);
-            T rt = shfl_idx<T>(incl, 31);
-            // incoming prefix of this lane's row segment, warp-local
-            T in = SEG ? seg_fold<Op>(run, lf, lin) : Op::apply(run, lin);
-            bool inf = SEG && (f || lf);
-            T r2 = in;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                if (SEG && ((hd >> k) & 1u)) { r2 = Op::identity(); inf = true; }
-                if (EXCL) { y[j].v[k] = r2; r2 = Op::apply(r2, x.v[k]); }
-                else      { r2 = Op::apply(r2, x.v[k]); y[j].v[k] = r2; }
-                if (SEG && inf) fm |= 1u << (4 * j + k);
-            }
-            run = SEG ? seg_fold<Op>(run, hm != 0u, rt) : Op::apply(run, rt);
-            f = f || (hm != 0u);
-        }
-        wtot = run; wfl = f;
-    }
-    // wp/wpf: prefix of the warps before this one in the tile; cin: carry into the tile
-    template <bool SEG>
-    __device__ __forceinline__ void emit(T* out, int64_t gidx, int64_t limit, bool fast, bool vec,
-                                         T wp, bool wpf, T cin) const {
-        const int lane = lane_id();
-        const T cw = Op::apply(cin, wp);
-#pragma unroll
-        for (int j = 0; j < V; ++j) {
-            Row4<T> o;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                const T yk = y[j].v[k];
-                if constexpr (Op::kSplitDesc) {            // f32 add: carry added last
-                    T loc = Op::apply(wp, yk);
-                    if (SEG && ((fm >> (4 * j + k)) & 1u)) o.v[k] = yk;
-                    else if (SEG && wpf) o.v[k] = loc;
-                    else o.v[k] = Op::apply(cin, loc);
-                } else {
-                    if (SEG && ((fm >> (4 * j + k)) & 1u)) o.v[k] = yk;
-                    else if (SEG && wpf) o.v[k] = Op::apply(wp, yk);
-                    else o.v[k] = Op::apply(cw, yk);
-                }
-            }
-            const int64_t idx = gidx + j * 128 + lane * 4;
-            if (fast) st_stream_v4(out + idx, row_to_u4<T>(o));
-            else store_row<Op>(out, idx, limit, vec, o);
-        }
-    }
-};
-
 // The same engine with the segmentation chosen per call (SEG is a per-tile runtime property
 // in the pipelined kernel, which keeps the state of two tiles in flight per warp).
 template <class Op, int V>

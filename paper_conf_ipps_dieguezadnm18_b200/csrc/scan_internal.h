@@ -19,6 +19,17 @@ struct NvtxRange {
     NvtxRange& operator=(const NvtxRange&) = delete;
 };
 
+// ---------------------------------------------------------------- launch facts (scan_launch.cu)
+// SM count of the current device, and per (device, kernel): the dynamic shared memory /
+// non-portable cluster opt-ins plus the occupancy -- cached per device, thread-safe.
+cudaError_t current_device_sms(int* sms);
+cudaError_t kernel_prepare(const void* func, int threads, size_t dyn_smem, bool nonportable_cluster, int* occ);
+// Persistent grid of min(occupancy x SMs, tiles) CTAs launched COOPERATIVELY (the whole
+// grid co-resident, as the static round-robin tile schedules require), optionally as a
+// programmatic dependent of the stream's previous kernel.
+cudaError_t launch_persistent(const void* func, void** args, int64_t tiles, int threads, size_t dyn_smem,
+                              bool pdl, cudaStream_t s);
+
 enum class OpCode : int { AddU32 = 0, MaxI32 = 1, MaxU32 = 2, MaxF32 = 3, AddF32 = 4 };
 
 // ---------------------------------------------------------------- single-pass look-back
@@ -44,8 +55,8 @@ struct LookbackParams {
 // problem: packed 8-byte descriptors ~80 % of copy, 16-byte slots ~90 %, 32/64-byte ~99 %
 // (the look-back round trip under full HBM load was dominated by line contention).
 constexpr int kDescWords = 8;
-int64_t lookback_tile_elems(int variant);
-int lookback_num_variants();
+int64_t lookback_tile_elems(int variant);      // 0 for an unknown variant
+bool lookback_variant_valid(int variant);
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s);
 
 // ---------------------------------------------------------------- fused peer exchange

@@ -14,26 +14,25 @@
 // carry crosses problems.  Small N costs no extra launches and rows need not be 16-byte
 // aligned (only the base pointers).
 //
-// B200 structure of the default kernel (variant 0, lookback_pipelined_kernel):
-//   * persistent, one CTA per SM; tiles of 16384 elements (64 KiB) are assigned round robin
-//     (tile = cta + k * grid; blocks dispatch in index order, so every tile a CTA waits on
-//     belongs to a CTA that is already running);
-//   * a producer warp streams the CTA's tiles into a 3-stage shared-memory ring with 1-D
-//     TMA bulk copies (cp.async.bulk, SASS UBLKCP) completing on mbarriers -- the bytes in
-//     flight are bounded by shared memory, not by registers;
-//   * 16 consumer warps scan each staged tile in two passes over smem; right after pass 1
-//     the last consumer warp publishes the tile aggregate (A), so aggregates never wait for
-//     a look-back; consumers run pass 1 of tile i+1 before pass 2 of tile i;
-//   * a dedicated look-back warp resolves each tile's carry with a 160-tile window (M = 5
-//     descriptors per lane per round trip, one window >= one round of 148 tiles).
+// Variants (scan_batch_ex `param`; AUTO uses 1, 2 and 3, scan_autotune also tries 0, 10):
+//   3  lookback_l2_kernel -- the default for few large problems (G*N >= 2^22), configs[2]:
+//      persistent, one CTA per SM, tiles of 8192 elements (32 KiB) assigned round robin
+//      (tile = cta + k * grid, launched cooperatively so the whole grid is co-resident);
+//      every tile is read TWICE but from HBM once: read 1 (TMA bulk copy into a smem ring,
+//      SASS UBLKCP) feeds 4 reducer warps that publish the tile aggregate (A) at once and
+//      free the slot; 8 speculative look-back warps resolve the carry while the data waits
+//      in L2; read 2 (L2 -> smem) feeds 8 scanner warps that add the carry and store.
+//      The next round's read 1 is L2-prefetched (UBLKPF).  ~102 % of measured copy at 2^30.
+//   0/1 lookback_pipelined_kernel -- persistent, one read: a producer warp streams 64 / 32
+//      KiB tiles into a 3-slot TMA ring, 16 / 8 consumer warps scan each staged tile in two
+//      passes, a dedicated look-back warp resolves the carry (window of 160 / 128 tiles);
+//      the tile holds its smem slot until its carry arrives (Little's law: ~85-91 % of
+//      copy for one huge problem).  1 = the AUTO choice for small totals (< 2^22).
+//   2  lookback_tma_kernel -- one 8192-element tile per CTA in blockIdx order (in-order
+//      dispatch: every tile a CTA waits on belongs to a running CTA); short / unaligned rows.
+//   10 lookback_regtile_kernel -- one 8192-element register tile per CTA (no smem staging).
 // Measured limits (tools/trace_lookback.py): a descriptor round trip costs
-// ~2 us under full HBM load and a tile holds its smem slot from TMA issue to pass 2, so a
-// single 2^30-element problem runs at ~80 % of the measured copy bandwidth.
-// Other variants (kept measurable through scan_batch_ex `param`): 1 = 32 KiB tiles,
-// 2 = one tile per CTA (short / unaligned rows), 3 = L2-staged two-read form (limited by
-// L2 slice throughput on B200), 4 = two look-back warps, 5 = register-resident waiting
-// tiles, 10-12 = one register tile per CTA, 13/14 = thread-block clusters of 16/8 register
-// tiles that combine through DSMEM and look back per cluster (G = 1; G > 1 runs 10).
+// ~2 us under full HBM load; the L2-staged form keeps the waiting data in L2, not smem.
 //
 // Descriptors (one per tile; reset-free thanks to a 30-bit epoch tag in every word):
 //   word = payload32 << 32 | tag << 2 | status      status 0 X (not ready), 1 A, 2 P
@@ -43,12 +42,8 @@
 //   self-contained, so relaxed (.STRONG.GPU, L1-bypassing) accesses suffice.
 // The last CTA to finish resets the ticket / done counters and advances the epoch, so
 // consecutive launches (also CUDA-graph replays) need no memset.
-#include <cooperative_groups.h>
-
 #include "scan_common.cuh"
 #include "scan_internal.h"
-
-namespace cg = cooperative_groups;
 
 namespace scanb200 {
 
@@ -58,7 +53,6 @@ constexpr uint32_t ST_A = 1u, ST_P = 2u;
 constexpr uint32_t TAG_MASK = 0x3FFFFFFFu;
 constexpr int LB_M = 4;                      // descriptors per lane per look-back round trip
 
-int num_sms();
 
 __device__ __forceinline__ void st_relaxed_u64(uint64_t* p, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
@@ -263,84 +257,6 @@ __device__ __forceinline__ uint32_t read_tag(const LookbackParams& p) {
     return (e + 1u) & TAG_MASK;
 }
 
-
-// ---------------------------------------------------------------- persistent, warp-specialised
-template <class Op, int WARPS, int V, int S>
-__global__ void __launch_bounds__((WARPS + 1) * 32) lookback_persistent_kernel(LookbackParams p, int64_t num_tiles) {
-    using T = typename Op::T;
-    using C = typename Op::Carry;
-    constexpr int TILE = WARPS * 32 * V * 4;
-    extern __shared__ __align__(128) unsigned char dsm[];
-    T* s_data = (T*)dsm;
-    __shared__ uint64_t s_full[S], s_empty[S];
-    __shared__ int64_t s_tid[S], s_r[S];
-    __shared__ uint32_t s_seg[S], s_fast[S];
-    __shared__ uint32_t s_tag;
-    __shared__ C s_carry;
-    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
-    __shared__ __align__(16) uint32_t s_wflag[(WARPS + 3) & ~3];
-    const int warp = threadIdx.x >> 5, lane = lane_id();
-
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int s = 0; s < S; ++s) { mbar_init(&s_full[s], 1); mbar_init(&s_empty[s], WARPS); }
-        fence_mbar_init();
-        s_tag = read_tag(p);
-    }
-    __syncthreads();
-    const uint32_t tag = s_tag;
-
-    if (warp == WARPS) {
-        // ---------------- producer warp: this CTA's tiles (round robin) into the TMA ring
-        const T* in = (const T*)p.in;
-        const uint64_t pol = l2_evict_first_policy();
-        int stage = 0;
-        uint32_t phase = 0;
-        for (int64_t t = blockIdx.x;; t += gridDim.x) {
-            mbar_wait(&s_empty[stage], phase ^ 1u);             // consumers freed this slot
-            if (t >= num_tiles) {
-                if (lane == 0) { s_tid[stage] = -1; mbar_arrive(&s_full[stage]); }
-                break;
-            }
-            const TileInfo ti = classify(p, t, TILE);
-            T* dst = s_data + (size_t)stage * TILE;
-            const int64_t base = t * (int64_t)TILE;
-            if (lane == 0) { s_tid[stage] = t; s_r[stage] = ti.r; s_seg[stage] = ti.seg; s_fast[stage] = ti.fast; }
-            if (ti.fast) {
-                if (lane == 0) {
-                    mbar_expect_tx(&s_full[stage], TILE * 4);
-                    tma_load_1d(dst, in + base, TILE * 4, &s_full[stage], pol);
-                }
-            } else {
-                // ragged tail tile or unaligned base pointers: guarded copy, identity padding
-                for (int i = lane; i < TILE; i += 32)
-                    dst[i] = base + i < p.total ? from_bits<T>(ld_stream_u32(in + base + i)) : Op::identity();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&s_full[stage]);
-            }
-            if (++stage == S) { stage = 0; phase ^= 1u; }
-        }
-    } else {
-        // ---------------- consumer warps
-        int stage = 0;
-        uint32_t phase = 0;
-        while (true) {
-            mbar_wait(&s_full[stage], phase);
-            const int64_t t = s_tid[stage];
-            if (t < 0) break;
-            const int64_t r = s_r[stage];
-            const bool fast = s_fast[stage] != 0u;
-            const T* st = s_data + (size_t)stage * TILE;
-            if (s_seg[stage]) tile_body_smem<Op, true, WARPS, V, true>(p, t, tag, r, st, fast, &s_carry, s_wval, s_wflag);
-            else              tile_body_smem<Op, false, WARPS, V, true>(p, t, tag, r, st, fast, &s_carry, s_wval, s_wflag);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&s_empty[stage]);
-            if (++stage == S) { stage = 0; phase ^= 1u; }
-        }
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
-}
 
 // ---------------------------------------------------------------- pipelined, dedicated look-back warp
 // Warp roles: WARPS consumer warps, one producer warp (TMA ring), one look-back warp.
@@ -586,202 +502,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
     if (threadIdx.x == 0) epilogue(p);
 }
 
-// ---------------------------------------------------------------- register-resident pipeline
-// As the pipelined kernel, but pass 1 leaves each element's warp-local prefix in registers
-// (WarpTileR) and releases the shared-memory slot at once: smem only covers load + pass 1,
-// and the tiles waiting for their carry sit in the register file (two per consumer warp).
-// Per-tile headers live in their own ring (SH entries) released after the outputs are
-// written.  Roles: WARPS consumers | producer (TMA) | look-back warp.
-template <class Op, int WARPS, int V, int S, int SH, int M, int NST>
-__global__ void __launch_bounds__((WARPS + 2) * 32, 1) lookback_regs_kernel(LookbackParams p, int64_t num_tiles) {
-    using T = typename Op::T;
-    using C = typename Op::Carry;
-    constexpr int WCH = V * 128, TILE = WARPS * WCH;
-    extern __shared__ __align__(128) unsigned char dsm[];
-    T* data = (T*)dsm;
-    __shared__ SlotHdr<Op, WARPS> s_hdr[SH];
-    __shared__ uint64_t fullR[S], emptyR[S], p1[SH], cr[SH], emptyH[SH];
-    __shared__ uint32_t s_tag;
-    const int warp = threadIdx.x >> 5, lane = lane_id();
-
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < S; ++s) { mbar_init(&fullR[s], 1); mbar_init(&emptyR[s], WARPS); }
-        for (int s = 0; s < SH; ++s) { mbar_init(&p1[s], 1); mbar_init(&cr[s], 1); mbar_init(&emptyH[s], WARPS); }
-        fence_mbar_init();
-        s_tag = read_tag(p);
-    }
-    __syncthreads();
-    const uint32_t tag = s_tag;
-    const bool excl = p.exclusive;
-
-    if (warp < WARPS) {
-        // ---------------- consumers
-        WarpTileR<Op, V> A, B;
-        auto pass1 = [&](WarpTileR<Op, V>& st, int64_t i) -> bool {
-            const int sR = (int)(i % S), sH = (int)(i % SH);
-            mbar_wait(&fullR[sR], (uint32_t)((i / S) & 1));
-            SlotHdr<Op, WARPS>& h = s_hdr[sH];
-            if (h.tid < 0) {
-                if (warp == WARPS - 1 && lane == 0) mbar_arrive(&p1[sH]);
-                return false;
-            }
-            if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 0);
-            const T* srow = data + (size_t)sR * TILE + warp * WCH;
-            const int64_t r = h.r;
-            if (h.seg) {
-                const bool small = p.N < TILE;
-                const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
-                if (excl) st.template pass1<true, true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
-                else      st.template pass1<true, false>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
-            } else {
-                if (excl) st.template pass1<false, true>(srow, warp * WCH, false, 0u, 1u, -1);
-                else      st.template pass1<false, false>(srow, warp * WCH, false, 0u, 1u, -1);
-            }
-            __threadfence_block();
-            __syncwarp();
-            if (lane == 0) {
-                mbar_arrive(&emptyR[sR]);                 // the tile now lives in registers
-                h.wtot[warp] = st.wtot;
-                h.wfl[warp] = st.wfl ? 1u : 0u;
-            }
-            consumer_bar(WARPS * 32);
-            if (warp == WARPS - 1) {
-                const bool seg = h.seg != 0u;
-                T run = Op::identity(); bool f = false;
-#pragma unroll
-                for (int w = 0; w < WARPS; ++w) {
-                    if (lane == w) { h.wp[w] = run; h.wpf[w] = f ? 1u : 0u; }
-                    const T v = h.wtot[w];
-                    const bool fw = seg && h.wfl[w] != 0u;
-                    run = fw ? v : Op::apply(run, v);
-                    f = f || fw;
-                }
-                const bool has_head = seg ? f : (r == 0);
-                if (lane == 0) {
-                    h.agg = Op::to_carry(run);
-                    h.has_head = has_head ? 1u : 0u;
-                    trace_stamp(p, h.tid, 1);
-                    Desc<Op>::publish(p, h.tid, tag, has_head ? ST_P : ST_A, h.agg);
-                }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&p1[sH]);
-            }
-            return true;
-        };
-        auto pass2 = [&](const WarpTileR<Op, V>& st, int64_t i) {
-            const int sH = (int)(i % SH);
-            mbar_wait(&cr[sH], (uint32_t)((i / SH) & 1));
-            const SlotHdr<Op, WARPS>& h = s_hdr[sH];
-            const int64_t gidx = h.tid * (int64_t)TILE + warp * WCH;
-            const T cin = Op::from_carry(h.carry);
-            const T wp = h.wp[warp];
-            const bool wpf = h.wpf[warp] != 0u, fast = h.fast != 0u;
-            if (h.seg) st.template emit<true>((T*)p.out, gidx, p.total, fast, p.vec, wp, wpf, cin);
-            else       st.template emit<false>((T*)p.out, gidx, p.total, fast, p.vec, wp, wpf, cin);
-            __syncwarp();
-            if (lane == 0) {
-                if (warp == 0) trace_stamp(p, h.tid, 3);
-                mbar_arrive(&emptyH[sH]);
-            }
-        };
-        // (a third register state would let consumers run two tiles ahead, but at 448
-        //  threads ptxas caps the kernel at 128 registers and it spills: measured slower)
-        static_assert(NST == 2, "two register states per consumer warp");
-        int64_t i = 0;
-        if (pass1(A, 0)) {
-            while (true) {
-                ++i;
-                bool more = pass1(B, i);
-                pass2(A, i - 1);
-                if (!more) break;
-                ++i;
-                more = pass1(A, i);
-                pass2(B, i - 1);
-                if (!more) break;
-            }
-        }
-    } else if (warp == WARPS) {
-        // ---------------- producer: this CTA's tiles (round robin) into the TMA ring
-        const T* in = (const T*)p.in;
-        const uint64_t pol = l2_evict_first_policy();
-        int64_t i = 0;
-        for (int64_t t = blockIdx.x;; t += gridDim.x, ++i) {
-            const int sR = (int)(i % S), sH = (int)(i % SH);
-            mbar_wait(&emptyR[sR], (uint32_t)((i / S) & 1) ^ 1u);
-            mbar_wait(&emptyH[sH], (uint32_t)((i / SH) & 1) ^ 1u);
-            SlotHdr<Op, WARPS>& h = s_hdr[sH];
-            if (t >= num_tiles) {
-                if (lane == 0) { h.tid = -1; mbar_arrive(&fullR[sR]); }
-                break;
-            }
-            const TileInfo ti = classify(p, t, TILE);
-            T* dst = data + (size_t)sR * TILE;
-            const int64_t base = t * (int64_t)TILE;
-            if (lane == 0) { h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast; }
-            if (ti.fast) {
-                if (lane == 0) {
-                    mbar_expect_tx(&fullR[sR], TILE * 4);
-                    tma_load_1d(dst, in + base, TILE * 4, &fullR[sR], pol);
-                }
-            } else {
-                for (int k = lane; k < TILE; k += 32)
-                    dst[k] = base + k < p.total ? from_bits<T>(ld_stream_u32(in + base + k)) : Op::identity();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&fullR[sR]);
-            }
-        }
-    } else {
-        // ---------------- look-back warp (speculative: starts before the tile's pass 1)
-        for (int64_t i = 0;; ++i) {
-            const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
-            if (t >= num_tiles) break;
-            const int sH = (int)(i % SH);
-            C carry = Op::cidentity();
-            uint32_t stats[2] = {0u, 0u};
-            if (lane == 0) trace_stamp(p, t, 4);
-            if (((t * (int64_t)TILE) % p.N) != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
-            mbar_wait(&p1[sH], (uint32_t)((i / SH) & 1));
-            SlotHdr<Op, WARPS>& h = s_hdr[sH];
-            if (lane == 0) {
-                if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
-                h.carry = carry;
-                trace_stamp(p, t, 2);
-                trace_value(p, t, 5, stats[0]);
-                trace_value(p, t, 6, stats[1]);
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&cr[sH]);
-        }
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
-}
-
-template <class Op, int WARPS, int V, int S, int SH, int M, int NST>
-cudaError_t launch_regs(const LookbackParams& p, cudaStream_t s) {
-    constexpr int TILE = WARPS * V * 128;
-    constexpr int SMEM = S * TILE * 4;
-    constexpr int THREADS = (WARPS + 2) * 32;
-    auto kern = lookback_regs_kernel<Op, WARPS, V, S, SH, M, NST>;
-    static int occ = 0;
-    if (occ == 0) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-        if (e != cudaSuccess) return e;
-        int o = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
-        if (e != cudaSuccess) return e;
-        if (o < 1) return cudaErrorInvalidConfiguration;
-        occ = o;
-    }
-    const int64_t tiles = (p.total + TILE - 1) / TILE;
-    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    int64_t grid = (int64_t)occ * num_sms();
-    if (grid > tiles) grid = tiles;
-    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
-    return cudaGetLastError();
-}
-
-// ---------------------------------------------------------------- two reads, L2-staged (variant 0)
+// ---------------------------------------------------------------- two reads, L2-staged (variant 3)
 // Little's law: a tile that waits in shared memory for its carry holds a slot for the
 // whole look-back latency (several us under full HBM load), which caps a single huge
 // problem at ~5 TB/s.  Here the tile is read TWICE but from HBM only once:
@@ -1030,31 +751,10 @@ cudaError_t launch_l2(const LookbackParams& p, cudaStream_t s) {
     constexpr int SMEM = (SR + SW) * TILE * 4;
     constexpr int THREADS = (NS + NR + 2 + NLB) * 32;
     auto kern = lookback_l2_kernel<Op, NS, NR, SR, SW, SH, M, NLB>;
-    static int occ = 0;
-    if (occ == 0) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-        if (e != cudaSuccess) return e;
-        int o = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
-        if (e != cudaSuccess) return e;
-        if (o < 1) return cudaErrorInvalidConfiguration;
-        occ = o;
-    }
-    const int64_t tiles = (p.total + TILE - 1) / TILE;
-    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    int64_t grid = (int64_t)occ * num_sms();
-    if (grid > tiles) grid = tiles;
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)grid, 1, 1);
-    cfg.blockDim = dim3(THREADS, 1, 1);
-    cfg.dynamicSmemBytes = SMEM;
-    cfg.stream = s;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = p.pdl_first ? 1 : 0;
-    return cudaLaunchKernelEx(&cfg, kern, p, tiles);
+    int64_t tiles = (p.total + TILE - 1) / TILE;
+    LookbackParams pc = p;
+    void* args[] = {&pc, &tiles};
+    return launch_persistent((const void*)kern, args, tiles, THREADS, SMEM, p.pdl_first, s);
 }
 
 // ---------------------------------------------------------------- one tile per CTA (comparison)
@@ -1184,108 +884,15 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackPa
     if (threadIdx.x == 0) epilogue(p);
 }
 
-// ---------------------------------------------------------------- clustered look-back
-// One problem (G = 1) of a few 2^20 elements, latency bound (configs[0]).  CS CTAs of one
-// register tile each form a thread-block cluster; the cluster first combines its CTA
-// aggregates through distributed shared memory (one cluster barrier), then only the
-// CLUSTER takes part in the decoupled look-back: descriptor q is cluster q's aggregate /
-// inclusive prefix, so 2^20 elements need 8 descriptors (one look-back round trip) instead
-// of 128.  Clusters follow blockIdx (in-order dispatch).  Every CTA's last warp runs the
-// (identical) look-back itself, so no second cluster barrier is needed; rank 0 publishes.
-template <class Op, int WARPS, int V, int CS>
-__global__ void __launch_bounds__(WARPS * 32) lookback_cluster_kernel(LookbackParams p) {
-    using T = typename Op::T;
-    using C = typename Op::Carry;
-    constexpr int TILE = WARPS * 32 * V * 4, WCH = V * 128;
-    __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
-    __shared__ C s_agg, s_carry;
-    cg::cluster_group cl = cg::this_cluster();
-    const unsigned crank = cl.block_rank();
-    const int64_t q = (int64_t)blockIdx.x / CS;
-    const int warp = threadIdx.x >> 5, lane = lane_id();
-    const uint32_t tag = read_tag(p);
-    const int64_t wb = (int64_t)blockIdx.x * TILE + warp * WCH;
-    WarpTile<Op, false, V> wt;
-    wt.load((const T*)p.in, wb, p.total, p.vec);
-    wt.scan();
-    if (lane == 0) s_wval[warp] = wt.wtot;
-    __syncthreads();
-    T wp = Op::identity();
-#pragma unroll
-    for (int w = 0; w < WARPS; ++w)
-        if (w < warp) wp = Op::apply(wp, s_wval[w]);
-    if (warp == WARPS - 1 && lane == 0) s_agg = Op::to_carry(Op::apply(wp, wt.wtot));
-    cl.sync();
-    C a = Op::cidentity();
-    if (lane < CS) a = *cl.map_shared_rank(&s_agg, (unsigned)lane);
-    const C pre = warp_reduce_carry<Op>((unsigned)lane < crank ? a : Op::cidentity());
-    // done with the peers' shared memory: arrive now, wait before exiting
-    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-    if (warp == WARPS - 1) {
-        const C ctot = warp_reduce_carry<Op>(a);
-        if (crank == 0 && lane == 0) Desc<Op>::publish(p, q, tag, q == 0 ? ST_P : ST_A, ctot);
-        C carry = Op::cidentity();
-        if (q > 0) carry = look_back<Op>(p, q, tag);
-        if (lane == 0) {
-            if (crank == 0 && q > 0) Desc<Op>::publish(p, q, tag, ST_P, Op::capply(carry, ctot));
-            s_carry = carry;
-        }
-    }
-    __syncthreads();
-    wt.store((T*)p.out, wb, p.total, p.vec, wp, false, Op::from_carry(Op::capply(s_carry, pre)), p.exclusive);
-    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-    __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
-}
-
 // ---------------------------------------------------------------- launchers
-int g_num_sms = 0;
-
-int num_sms() {
-    if (g_num_sms == 0) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-        if (g_num_sms <= 0) g_num_sms = 148;
-    }
-    return g_num_sms;
-}
-
-template <class Op, int WARPS, int V, int S>
-cudaError_t launch_persistent(const LookbackParams& p, cudaStream_t s) {
-    constexpr int TILE = WARPS * 32 * V * 4;
-    constexpr int SMEM = S * TILE * 4;
-    constexpr int THREADS = (WARPS + 1) * 32;
-    auto kern = lookback_persistent_kernel<Op, WARPS, V, S>;
-    static int occ = 0;                       // per instantiation; computed once
-    if (occ == 0) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-        if (e != cudaSuccess) return e;
-        int o = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
-        if (e != cudaSuccess) return e;
-        if (o < 1) return cudaErrorInvalidConfiguration;
-        occ = o;
-    }
-    const int64_t tiles = (p.total + TILE - 1) / TILE;
-    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    int64_t grid = (int64_t)occ * num_sms();
-    if (grid > tiles) grid = tiles;
-    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
-    return cudaGetLastError();
-}
-
 template <class Op, int WARPS, int V>
 cudaError_t launch_tma(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
     constexpr int SMEM = TILE * 4;
     const int64_t tiles = (p.total + TILE - 1) / TILE;
     if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    if (SMEM > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(lookback_tma_kernel<Op, WARPS, V>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-        if (e != cudaSuccess) return e;
-    }
+    cudaError_t e = kernel_prepare((const void*)lookback_tma_kernel<Op, WARPS, V>, WARPS * 32, SMEM, false, nullptr);
+    if (e != cudaSuccess) return e;
     lookback_tma_kernel<Op, WARPS, V><<<(unsigned)tiles, WARPS * 32, SMEM, s>>>(p);
     return cudaGetLastError();
 }
@@ -1299,56 +906,16 @@ cudaError_t launch_regtile(const LookbackParams& p, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-template <class Op, int WARPS, int V, int CS>
-cudaError_t launch_lb_cluster(const LookbackParams& p, cudaStream_t s) {
-    if (p.N != p.total) return launch_regtile<Op, WARPS, V>(p, s);   // G > 1: per-tile look-back
-    constexpr int TILE = WARPS * 32 * V * 4;
-    auto kern = lookback_cluster_kernel<Op, WARPS, V, CS>;
-    static bool init = false;
-    if (!init) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (e != cudaSuccess) return e;
-        init = true;
-    }
-    const int64_t tiles = (p.total + TILE - 1) / TILE;
-    const int64_t grid = (tiles + CS - 1) / CS * CS;
-    if (grid > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)grid, 1, 1);
-    cfg.blockDim = dim3(WARPS * 32, 1, 1);
-    cfg.stream = s;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = CS;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, kern, p);
-}
-
 template <class Op, int WARPS, int V, int S, int M, int NLB, int PF = 0>
 cudaError_t launch_pipelined(const LookbackParams& p, cudaStream_t s) {
     constexpr int TILE = WARPS * 32 * V * 4;
     constexpr int SMEM = S * TILE * 4;
     constexpr int THREADS = (WARPS + 1 + NLB) * 32;
     auto kern = lookback_pipelined_kernel<Op, WARPS, V, S, M, NLB, PF>;
-    static int occ = 0;
-    if (occ == 0) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-        if (e != cudaSuccess) return e;
-        int o = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, THREADS, SMEM);
-        if (e != cudaSuccess) return e;
-        if (o < 1) return cudaErrorInvalidConfiguration;
-        occ = o;
-    }
-    const int64_t tiles = (p.total + TILE - 1) / TILE;
-    if (tiles > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
-    int64_t grid = (int64_t)occ * num_sms();
-    if (grid > tiles) grid = tiles;
-    kern<<<(unsigned)grid, THREADS, SMEM, s>>>(p, tiles);
-    return cudaGetLastError();
+    int64_t tiles = (p.total + TILE - 1) / TILE;
+    LookbackParams pc = p;
+    void* args[] = {&pc, &tiles};
+    return launch_persistent((const void*)kern, args, tiles, THREADS, SMEM, false, s);
 }
 
 template <class Op>
@@ -1358,27 +925,24 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1, 0>(p, s);   // 32 KiB tiles (small, L2-resident totals)
     case 2: return launch_tma<Op, 8, 8>(p, s);                     // one 8192-element tile per CTA
     case 3: return launch_l2<Op, 8, 4, 3, 3, 8, 5, 8>(p, s);       // two reads (L2-staged), 8-tile header ring, 8 look-back warps
-    case 4: return launch_pipelined<Op, 16, 8, 3, 5, 2, 1>(p, s);  // as 0 with two look-back warps
-    case 5: return launch_regs<Op, 12, 8, 4, 8, 5, 2>(p, s);       // register-resident waiting tiles, 48 KiB
-    case 6: return launch_tma<Op, 8, 4>(p, s);                     // one 4096-element tile per CTA
-    case 7: return launch_pipelined<Op, 8, 4, 4, 4, 1>(p, s);      // 16 KiB tiles, 4-slot ring
-    case 8: return launch_pipelined<Op, 18, 8, 3, 5, 1, 2>(p, s);  // 72 KiB tiles, L2 prefetch +2 rounds
     case 10: return launch_regtile<Op, 16, 4>(p, s);               // one 8192-element register tile per CTA
-    case 11: return launch_regtile<Op, 8, 4>(p, s);                // one 4096-element register tile per CTA
-    case 12: return launch_regtile<Op, 32, 4>(p, s);               // one 16384-element register tile per CTA
-    case 13: return launch_lb_cluster<Op, 16, 4, 16>(p, s);        // 16-CTA clusters of 8192-element tiles (G = 1)
-    case 14: return launch_lb_cluster<Op, 16, 4, 8>(p, s);         // 8-CTA clusters of 8192-element tiles (G = 1)
-    default: return launch_pipelined<Op, 16, 8, 3, 5, 1, 0>(p, s); // as 0 without the L2 prefetch
+    default: return cudaErrorInvalidValue;
     }
 }
 
 }  // namespace
 
-int64_t lookback_tile_elems(int variant) {
-    return (variant == 0 || variant == 4 || variant == 9 || variant == 12) ? 16384 : variant == 5 ? 12288
-         : variant == 8 ? 18432 : (variant == 6 || variant == 7 || variant == 11) ? 4096 : 8192;
+// Variants of the product library.  The research variants measured in round 1 (4-9 and
+// 11-14: two look-back warps, register-resident waiting tiles, 16/72 KiB tiles, one 4096 /
+// 16384-element tile per CTA, clustered look-back) were removed after they lost on every
+// shape (DESIGN.md §5 keeps their numbers); their ids stay unused.
+bool lookback_variant_valid(int variant) {
+    return variant == 0 || variant == 1 || variant == 2 || variant == 3 || variant == 10;
 }
-int lookback_num_variants() { return 15; }
+int64_t lookback_tile_elems(int variant) {
+    if (!lookback_variant_valid(variant)) return 0;
+    return variant == 0 ? 16384 : 8192;
+}
 
 cudaError_t launch_lookback(OpCode op, const LookbackParams& p, int variant, cudaStream_t s) {
     switch (op) {

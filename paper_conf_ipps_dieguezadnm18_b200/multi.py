@@ -83,6 +83,12 @@ def exchange_totals(totals: torch.Tensor, group=None) -> torch.Tensor:
     """All-gather this rank's G total slots (int64) into a rank-major [W, G] tensor."""
     world = dist.get_world_size(group)
     src = totals.contiguous().view(-1)
+    if src.is_cuda and dist.get_backend(group) == "gloo":
+        # gloo gathers host tensors only: stage the W*G*8 bytes through the host (plumbing
+        # for CPU-backed groups, e.g. several ranks sharing one GPU in tests)
+        out = torch.empty(world * src.numel(), dtype=totals.dtype)
+        dist.all_gather_into_tensor(out, src.cpu(), group=group)
+        return out.to(totals.device).view((world,) + tuple(totals.shape))
     out = torch.empty(world * src.numel(), dtype=totals.dtype, device=totals.device)
     dist.all_gather_into_tensor(out, src, group=group)
     return out.view((world,) + tuple(totals.shape))

@@ -49,3 +49,22 @@ def assert_parity(got: np.ndarray, x: np.ndarray, op: str, kind: str, label: str
             i = np.argwhere(bad)[0]
             raise AssertionError("%s mismatch at %s: got %r ref %r (%d bad)" % (
                 label, tuple(i), got[tuple(i)], ref[tuple(i)], int(bad.sum())))
+
+
+def spin_lib():
+    """Build (once, in-tree, nvcc for sm_100a) and load tests/c/libspin.so, the SM-occupying
+    spin kernel of tests/test_gpu_safety.py (test infrastructure, not the product)."""
+    import ctypes
+    import os
+    import subprocess
+    here = os.path.join(os.path.dirname(os.path.abspath(__file__)), "c")
+    src, so = os.path.join(here, "spin.cu"), os.path.join(here, "libspin.so")
+    if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+        tmp = so + ".tmp%d" % os.getpid()
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2",
+                               "-Xcompiler", "-fPIC", "-shared", "-o", tmp, src])
+        os.replace(tmp, so)
+    lib = ctypes.CDLL(so)
+    lib.spin_launch.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_ulonglong, ctypes.c_void_p]
+    lib.spin_launch.restype = ctypes.c_int
+    return lib

@@ -29,7 +29,7 @@ def test_library_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(_lib.lib, name), name
     assert set(_lib.EXPORTS) == declared
-    assert _lib.lib.scan_abi_version() == 2
+    assert _lib.lib.scan_abi_version() == 3
 
 
 def test_status_strings():
@@ -91,13 +91,14 @@ def test_binding_fails_loudly_without_library(tmp_path, monkeypatch):
         spec.loader.exec_module(mod)
 
 
-def test_lookback_variant_count_matches_library():
+def test_lookback_variants_match_library():
     # the binding, the library source and tests/test_gpu_parity.py::test_lookback_variants
-    # must agree on how many look-back variants exist
+    # must agree on which look-back variants exist
     import re
     from paper_conf_ipps_dieguezadnm18_b200 import _lib
     src = open(os.path.join(PKG, "csrc", "scan_lookback.cu")).read()
-    n = int(re.search(r"int lookback_num_variants\(\) \{ return (\d+); \}", src).group(1))
-    assert _lib.lib_num_lookback_variants() == n
+    body = re.search(r"bool lookback_variant_valid\(int variant\) \{\s*return ([^;]*);", src).group(1)
+    valid = tuple(sorted(int(v) for v in re.findall(r"variant == (\d+)", body)))
+    assert _lib.LOOKBACK_VARIANTS == valid
     par = open(os.path.join(os.path.dirname(__file__), "test_gpu_parity.py")).read()
-    assert '@pytest.mark.parametrize("variant", range(%d))\ndef test_lookback_variants' % n in par
+    assert '@pytest.mark.parametrize("variant", _lib.LOOKBACK_VARIANTS)\ndef test_lookback_variants' in par

@@ -20,7 +20,7 @@ def test_random_cases(seed):
     algos = [("auto", -1), ("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0), ("three_stage", 3),
              ("packed_warp", -1), ("packed_warp", 300), ("cluster", -1), ("cluster", 32 + 8),
              ("cluster", 64 + 2), ("cluster", 16)] + \
-            [("lookback", v) for v in range(_lib.lib_num_lookback_variants())]
+            [("lookback", v) for v in _lib.LOOKBACK_VARIANTS]
     for case in range(40):
         N = rng.choice([rng.randint(1, 300), rng.randint(300, 20000), rng.randint(20000, 400000)])
         G = rng.choice([1, 1, 2, rng.randint(1, 40), rng.randint(100, 5000)])

@@ -1,0 +1,55 @@
+"""Full-size single-GPU configurations beyond round 1's coverage, checked in full.
+
+* One int32 / uint32 problem of N = 2^31 + 4099 elements (8 GiB in + 8 GiB out) through the
+  AUTO path (the L2-staged look-back): tile and element indices beyond 2^31, a ragged last
+  tile, 8-byte descriptors; every output element against the streaming oracle.
+* configs[2]'s shape in int32 (G = 1, N = 2^30), inclusive and exclusive.
+The north_star asks for N "from 2^10 to beyond one GPU's HBM" (the sharded path covers the
+latter); PAPER.md:96 defines the problem for any N.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_ipps_dieguezadnm18_b200 as sb
+from gpu_util import device_inputs, to_host
+
+pytestmark = pytest.mark.gpu
+
+
+def _check_streamed(xd, out, kind, dtype, label):
+    so = oracle.StreamAdd(dtype, kind)
+    n = xd.numel()
+    step = 1 << 26
+    for a in range(0, n, step):
+        ref = so.feed(to_host(xd[a: a + step], dtype))
+        got = to_host(out[a: a + step], dtype)
+        if not np.array_equal(got, ref):
+            i = int(np.argmax(got != ref))
+            raise AssertionError("%s: chunk %d, first bad element %d: got %r ref %r" % (
+                label, a // step, a + i, got[i], ref[i]))
+
+
+@pytest.mark.parametrize("dist,kind", [("i32", "inclusive"), ("u32", "exclusive")])
+def test_single_problem_beyond_2e31_elements(dist, kind):
+    N = (1 << 31) + 4099
+    dtype = np.int32 if dist == "i32" else np.uint32
+    xd = device_inputs(dist, N, 0x5CA2018 + 9)
+    assert sb.plan(xd) == ("lookback", 3)
+    out = sb.scan(xd, "add", kind)
+    torch.cuda.synchronize()
+    _check_streamed(xd, out, kind, dtype, "N=2^31+4099 %s %s" % (dist, kind))
+    del xd, out
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("kind", ["inclusive", "exclusive"])
+def test_c3_shape_int32_full(kind):
+    N = 1 << 30
+    xd = device_inputs("i32", N, 0x5CA2018 + 3)
+    out = sb.scan(xd, "add", kind)
+    torch.cuda.synchronize()
+    _check_streamed(xd, out, kind, np.int32, "int32 N=2^30 %s" % kind)
+    del xd, out
+    torch.cuda.empty_cache()

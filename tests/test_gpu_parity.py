@@ -11,6 +11,7 @@ import torch
 import inputs
 import oracle
 import paper_conf_ipps_dieguezadnm18_b200 as sb
+from paper_conf_ipps_dieguezadnm18_b200 import _lib
 from gpu_util import COMBOS, DIST, NP, TORCH, assert_parity, device_inputs, to_device, to_host
 
 pytestmark = pytest.mark.gpu
@@ -39,7 +40,7 @@ def test_shapes_all_algos(algo, op, dt, kind):
             assert_parity(got, x, op, kind, label="%s %s %s %s N=%d G=%d" % (algo, op, dt, kind, N, G))
 
 
-@pytest.mark.parametrize("variant", range(15))
+@pytest.mark.parametrize("variant", _lib.LOOKBACK_VARIANTS)
 def test_lookback_variants(variant):
     for op, dt in COMBOS:
         for N, G in [(1, 3000), (3, 5000), (100, 333), (8193, 5), (65536 + 17, 3), (1 << 20, 1)]:
@@ -350,9 +351,13 @@ def test_autotune_table():
         x = inputs.generate("i32", G * N, seed=G + N).reshape(G, N)
         xd = to_device(x)
         before = sb.plan(xd)
+        before_max = sb.plan(xd, op="max", kind="exclusive")
         algo, param, us = sb.autotune(xd, "add", "inclusive")
         assert algo in sb.ALGOS and algo != "auto" and us > 0.0
         assert sb.plan(xd) == (algo, param)
+        # the tuned choice applies to (op, dtype, kind) it was measured on only
+        assert sb.plan(xd, op="max", kind="exclusive") == before_max
+        assert sb.plan(xd.view(torch.float32)) == before
         for op, dt in COMBOS:
             xx = inputs.generate(DIST[dt], G * N, seed=3 * G + N).reshape(G, N)
             for kind in ("inclusive", "exclusive"):

@@ -16,7 +16,7 @@ quick = "--quick" in sys.argv
 shapes = [(20000, 3), (70001, 1), (1000, 40)] if not quick else [(70001, 1), (1000, 5)]
 cases = [("cascade_cta", -1), ("cascade_warp", -1), ("three_stage", 0), ("packed_warp", -1),
          ("cluster", -1), ("cluster", 32 + 4), ("cluster", 2)] + \
-        [("lookback", v) for v in range(_lib.lib_num_lookback_variants())]
+        [("lookback", v) for v in _lib.LOOKBACK_VARIANTS]
 for dt, dist in (("i32", "i32"), ("f32", "f32s")):
     for N, G in shapes:
         x = torch.empty(N * G, dtype=torch.int32, device="cuda")
