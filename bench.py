@@ -5,22 +5,37 @@ Metric (BASELINE.json): Gelem/s (and % of the HBM roofline) of int32/f32 scans a
 GPUs.  Workload at N=1 = configs[1]: G = 4096 problems of N = 2^14 elements; one STEP is
 the four scans that config names -- add-scan of int32 and of f32, inclusive and exclusive
 -- each over the whole 2^26-element batch (256 MiB in + 256 MiB out per scan, larger
-than the 126 MB L2, so no flush is needed between steps).  Under torchrun (--gpus N > 1)
-every rank scans its own G = 4096 problems (problems mode, Case 1 of PAPER.md:191-193, no
-collective on the data path): weak scaling, value = elements of all ranks / max-over-ranks
-time.
+than the 126 MB L2, so no flush is needed between steps).  With --gpus N > 1 every rank
+scans its own G = 4096 problems (problems mode, Case 1 of PAPER.md:191-193, no collective
+on the data path): weak scaling, value = elements of all ranks / max-over-ranks time.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--no-extras] [--sweep]
+                    [--no-extras] [--no-e2e] [--no-cpu] [--sweep] [--dry-run]
 
+--gpus N > 1 without torchrun: bench.py re-launches itself under torch.distributed.run with
+N processes (one per GPU, 127.0.0.1 rendezvous); under torchrun WORLD_SIZE must equal N.
+Beside the headline line (rank 0 prints it) the legs the paper's multi-GPU figures need:
+  elements_mode_sharded_problem  configs[4]: one int32 problem, 2^33 elements per rank,
+                                 Stage 1+2 -> exchange -> Stage 3, with E_W and E_naive
+                                 (SURVEY §8(e)) and the NCCL / fused-peer exchange times;
+  scan_mps                       the paper's flagship Scan-MPS workload (PAPER.md:197-199,
+                                 249 [Fig. 9]): G = 2^28/N problems, each split over the W
+                                 ranks, n = 13, 20, 28;
+  c4_problems_mode               configs[3], strong scaling by problems;
+  roofline_c3 / extras           (W = 1) configs[2] with its own kernel roofline, ncu
+                                 traffic and oracle baseline; configs[0] warm and L2-flushed.
 `--impl reference` times the CPU oracle (the only reference this paper-only run has) on
-host cores, on a bounded sample of the same workload.
+host cores, on a bounded sample of the same workload.  `--dry-run` exercises only the rank
+plumbing (spawn, gloo process group, barriers, max over ranks) on a CPU-only host.
 """
 from __future__ import annotations
 
 import argparse
+import glob
+import hashlib
 import json
 import os
+import socket
 import statistics
 import sys
 import threading
@@ -40,6 +55,7 @@ VARIANTS = [("i32", "add", "inclusive"), ("i32", "add", "exclusive"),
 DIST = {"i32": "i32", "f32": "f32u"}
 TDT = {"i32": torch.int32, "f32": torch.float32}
 NPDT = {"i32": np.int32, "f32": np.float32}
+NOMINAL_HBM_GBS = 8000.0          # north_star "~8 TB/s peak"
 
 
 def _peaks():
@@ -50,6 +66,37 @@ def _peaks():
     return 6650.0, "fallback (B200_PROFILING.md)", {}
 
 
+def source_sha256() -> str:
+    """Hash of the library's sources (kernels, C-ABI, header): a committed ncu capture is
+    reported as this run's traffic only when it was taken on the same sources."""
+    h = hashlib.sha256()
+    files = sorted(glob.glob(os.path.join(ROOT, "paper_conf_ipps_dieguezadnm18_b200", "csrc", "*")) +
+                   glob.glob(os.path.join(ROOT, "include", "*.h")))
+    for f in files:
+        h.update(os.path.basename(f).encode())
+        h.update(open(f, "rb").read())
+    return h.hexdigest()
+
+
+def traffic_for(case: str):
+    """DRAM bytes (read + write) per launch of the dominant kernel of `case` from the ncu
+    capture profiles/ncu_traffic.json (tools/ncu_traffic.py), if its source hash matches."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None, "no capture"
+    try:
+        d = json.load(open(p))
+    except Exception as e:  # noqa: BLE001
+        return None, "unreadable capture: %r" % (e,)
+    if d.get("src_sha256") != source_sha256():
+        return None, "stale capture (library sources changed since %s)" % d.get("captured", "?")
+    e = d.get("cases", {}).get(case)
+    if not e:
+        return None, "case not captured"
+    return float(e["dram_bytes_read"] + e["dram_bytes_write"]), "ncu --set full capture %s (%s, src %s)" % (
+        d.get("captured", "?"), e.get("kernel", "?"), d["src_sha256"][:12])
+
+
 # ---------------------------------------------------------------- multi-rank plumbing
 # SCANB200_BENCH_BACKEND=gloo + SCANB200_BENCH_ONE_GPU=1 run every rank on cuda:0 with a gloo
 # process group: a dry run of the multi-rank control flow (barriers, max over ranks, the
@@ -58,13 +105,55 @@ DIST_BACKEND = os.environ.get("SCANB200_BENCH_BACKEND", "nccl")
 ONE_GPU = os.environ.get("SCANB200_BENCH_ONE_GPU") == "1"
 
 
+def _free_port() -> int:
+    with socket.socket(socket.AF_INET, socket.SOCK_STREAM) as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def maybe_respawn(args) -> None:
+    """--gpus N > 1 outside torchrun: re-exec as `torch.distributed.run --nproc-per-node N`
+    (one process per GPU; rank 0 prints the line).  Under torchrun, WORLD_SIZE must be N."""
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is not None:
+        if int(world_env) != args.gpus and args.impl == "ours":
+            sys.stderr.write("bench.py: --gpus %d but WORLD_SIZE=%s (launch N ranks for --gpus N)\n"
+                             % (args.gpus, world_env))
+            raise SystemExit(2)
+        return
+    if args.gpus <= 1 or args.impl != "ours":
+        return
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % args.gpus,
+           "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), os.path.abspath(__file__)] + sys.argv[1:]
+    sys.stdout.flush()
+    sys.stderr.flush()
+    os.execv(sys.executable, cmd)
+
+
 def max_over_ranks(v: float, world: int) -> float:
+    return reduce_over_ranks(v, world, "max")
+
+
+def reduce_over_ranks(v: float, world: int, how: str = "max") -> float:
     if world == 1:
         return v
     dev = "cuda" if DIST_BACKEND == "nccl" else "cpu"
     t = torch.tensor([v], dtype=torch.float64, device=dev)
-    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    op = torch.distributed.ReduceOp.MAX if how == "max" else torch.distributed.ReduceOp.MIN
+    torch.distributed.all_reduce(t, op=op)
     return float(t.item())
+
+
+def align_ranks(world: int) -> None:
+    """Barrier, then a 1-element all-reduce on the launching stream: ranks
+    leave together and the device queue of each is aligned before its start event."""
+    if world == 1:
+        return
+    torch.distributed.barrier()
+    if DIST_BACKEND == "nccl":
+        t = torch.zeros(1, device="cuda")
+        torch.distributed.all_reduce(t)
+    torch.cuda.synchronize()
 
 
 def all_gather_totals(t: torch.Tensor, world: int) -> torch.Tensor:
@@ -72,11 +161,7 @@ def all_gather_totals(t: torch.Tensor, world: int) -> torch.Tensor:
     from paper_conf_ipps_dieguezadnm18_b200 import multi
     if world == 1:
         return t.view(1, -1)
-    if DIST_BACKEND == "nccl":
-        return multi.exchange_totals(t)
-    parts = [torch.empty_like(t, device="cpu") for _ in range(world)]
-    torch.distributed.all_gather(parts, t.cpu())
-    return torch.stack(parts).to(t.device)
+    return multi.exchange_totals(t)
 
 
 # ---------------------------------------------------------------- clocks during the timed region
@@ -141,34 +226,24 @@ def make_inputs(rank: int, device):
     return xs
 
 
-def step(sb, xs, outs, events=None):
+def step(sb, xs, outs):
     for i, (dt, op, kind) in enumerate(VARIANTS):
-        if events is not None:
-            events[i][0].record()
         sb.scan(xs[dt], op, kind, out=outs[i])
-        if events is not None:
-            events[i][1].record()
 
 
-def timed_steps(sb, xs, outs, K, per_launch=False):
-    """K steps between two events on the launching stream; optionally per-launch events."""
-    ev = None
-    if per_launch:
-        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-               for _ in VARIANTS] for _ in range(K)]
+def timed_steps(sb, xs, outs, K, world):
+    """K steps between two events on the launching stream (device time), and the host wall
+    clock around the same region (synchronize on both sides) as a cross-check."""
     s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    torch.cuda.synchronize()
+    align_ranks(world)
+    w0 = time.perf_counter()
     s0.record()
-    for k in range(K):
-        step(sb, xs, outs, ev[k] if ev else None)
+    for _ in range(K):
+        step(sb, xs, outs)
     s1.record()
     torch.cuda.synchronize()
-    total_ms = s0.elapsed_time(s1)
-    launch_ms = None
-    if ev:
-        launch_ms = [statistics.mean(ev[k][i][0].elapsed_time(ev[k][i][1]) for k in range(K))
-                     for i in range(len(VARIANTS))]
-    return total_ms, launch_ms
+    wall_ms = (time.perf_counter() - w0) * 1e3
+    return s0.elapsed_time(s1), wall_ms
 
 
 def kernel_times(sb, xs, outs, reps):
@@ -185,6 +260,26 @@ def kernel_times(sb, xs, outs, reps):
     return res
 
 
+def validate_step(xs, outs, rows=(0, 1, 1234, G_C2 - 1)):
+    """After the timed region: the outputs of the LAST timed step are checked against the
+    oracle on sampled problems of every variant (bit-exact for int32, north_star tolerance
+    for f32).  Test infrastructure only -- nothing timed depends on it."""
+    import oracle
+    bad = []
+    for i, (dt, op, kind) in enumerate(VARIANTS):
+        x = xs[dt][list(rows)].view(torch.int32).cpu().numpy().view(NPDT[dt])
+        got = outs[i][list(rows)].view(torch.int32).cpu().numpy().view(NPDT[dt])
+        if dt == "f32":
+            ref, sabs = oracle.scan(x, op, kind, with_abs=True)
+            ok = bool(np.all(np.abs(got.astype(np.float64) - ref) <= 1e-5 * sabs))
+        else:
+            ok = np.array_equal(got, oracle.scan(x, op, kind))
+        if not ok:
+            bad.append("%s %s %s" % (dt, op, kind))
+    return {"checked": "problems %s of every variant vs the oracle" % (list(rows),), "ok": not bad, "failed": bad}
+
+
+# ---------------------------------------------------------------- end to end (host buffers)
 def e2e(sb, world=1, K=3):
     """The same step through the public host-buffer API: pinned host in -> scan -> host out.
     Under torchrun every rank runs it at once on its own GPU (its own PCIe link); the time
@@ -281,6 +376,280 @@ def c4_problems(sb, dev, world, rank, reps=5):
             "scaling": "strong (fixed 2^32-element batch)", "kernel": kern}
 
 
+def _peer_comms(world, max_G):
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    comms = {"peer": multi.PeerComm(max_G) if world > 1 else multi.PeerComm.loopback(1, max_G)[0]}
+    if world > 1 and DIST_BACKEND == "nccl":
+        comms["nccl"] = multi.NativeComm()
+    return comms
+
+
+def _time_calls(fn, reps, world):
+    """Device time per call (events on the launching stream), max over ranks."""
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    align_ranks(world)
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    for _ in range(reps):
+        fn()
+    s1.record()
+    torch.cuda.synchronize()
+    return max_over_ranks(s0.elapsed_time(s1) / reps, world)
+
+
+def _time_alone(fn, reps):
+    """Device time per call of THIS rank's work with no other rank involved."""
+    for _ in range(2):
+        fn()
+    torch.cuda.synchronize()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    for _ in range(reps):
+        fn()
+    s1.record()
+    torch.cuda.synchronize()
+    return s0.elapsed_time(s1) / reps
+
+
+def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB200_BENCH_ELEMS_LOG2", "33")),
+                  reps=10):
+    """configs[4]: one int32 add-scan sharded by elements (Multi-GPU Problem Scattering,
+    PAPER.md:195-205): each rank owns a contiguous 2^33-element portion (32 GiB in + 32 GiB
+    out) of ONE problem -- at W = 8 the problem is configs[4]'s N = 2^36.  Stage 1+2 ->
+    exchange -> Stage 3.  Weak-scaled (N = W x 2^33).
+
+    Efficiency: every rank first times, ALONE, (a) the same two-pass
+    pipeline on its portion with no peer (t_1, the W = 1 reference of the same pipeline) and
+    (b) the best single-GPU single-pass scan of its portion (t_sp, AUTO dispatch).  Then
+    E_W = min_r t_1 / max_r t_W and E_naive = min_r t_sp / max_r t_W (= Gelem/s(W) /
+    (W x single-pass Gelem/s of N/W on one GPU); <= ~2/3 by the 12 vs 8 B/elem argument)."""
+    import inputs
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    x = torch.empty(n_local, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "i32", SEED + 5, offset=rank * n_local)
+    y = torch.empty_like(x)
+    # (a)/(b): this rank alone
+    solo = multi.PeerComm.loopback(1, 1)[0]
+    t1 = _time_alone(lambda: multi.scan_multi(x, "add", "inclusive", mode="elements", out=y, backend="peer",
+                                              comm=solo), reps)
+    solo.close()
+    t_sp = _time_alone(lambda: sb.scan(x, "add", "inclusive", out=y), reps)
+    kern_sp = "%s %s" % sb.plan(x, y)
+    # the W-rank call: fused exchange (Stage 2 pushes the totals into later ranks' HBM,
+    # Stage 3 waits on the device; no collective call) is the product path, NCCL beside it
+    comms = _peer_comms(world, 1)
+    times = {}
+    for name, c in comms.items():
+        times[name] = _time_calls(lambda: multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
+                                                           backend="peer" if name == "peer" else "native", comm=c),
+                                  reps, world)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    for c in comms.values():
+        c.close()
+    ms = times["peer"]
+    # per-phase breakdown (the paper's Fig. 14, PAPER.md:283-289): Stage 1+2 / exchange /
+    # Stage 3, events between the three steps of the torch-backend path
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+    ph = [0.0, 0.0, 0.0]
+    t = sb.shard_totals(x, "add")                 # warm-up (workspace growth), totals reused
+    torch.cuda.synchronize()
+    for _ in range(reps):
+        ev[0].record()
+        sb.shard_totals(x, "add", totals=t)
+        ev[1].record()
+        allt = all_gather_totals(t, world)
+        ev[2].record()
+        sb.shard_scan(x, allt, rank, world, "add", "inclusive", out=y)
+        ev[3].record()
+        torch.cuda.synchronize()
+        for k in range(3):
+            ph[k] += ev[k].elapsed_time(ev[k + 1]) / reps
+    t1_min = reduce_over_ranks(t1, world, "min")
+    tsp_min = reduce_over_ranks(t_sp, world, "min")
+    hbm, _, _ = _peaks()
+    per_gpu_gbs = 12.0 * n_local / (ms * 1e-3) / 1e9          # reduce pass (4 B) + scan pass (8 B)
+    del x, y
+    torch.cuda.empty_cache()
+    return {"N_total": world * n_local, "N_per_gpu": n_local, "ms": ms,
+            "Gelem/s": world * n_local / ms / 1e6, "per_gpu_GB/s_at_12B_per_elem": per_gpu_gbs,
+            "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
+            "E_W": t1_min / ms, "E_naive": tsp_min / ms,
+            "t1_same_pipeline_alone_ms": t1_min, "t_single_pass_alone_ms": tsp_min,
+            "single_pass_kernel": kern_sp,
+            "efficiency_def": "E_W = min_r t(two-pass pipeline on the rank's portion, alone) / max_r t(W-rank "
+                              "call); E_naive = min_r t(single-pass AUTO scan of the portion, alone) / max_r "
+                              "t(W-rank call) (SURVEY 8(e))",
+            "exchange": ("fused peer stores in the Stage 2/3 kernels (scan_comm_create_peer)" if world > 1
+                         else "none (W=1; the fused-exchange kernels run with no peers)"),
+            "ms_by_exchange": times,
+            "phases_ms_rank%d" % rank: {"stage1+2_reduce": ph[0], "exchange": ph[1], "stage3_scan": ph[2]}}
+
+
+def scan_mps(sb, dev, world, rank, logs=(13, 20, 28), reps=10):
+    """The paper's flagship Scan-MPS workload (PAPER.md:197-199, 249 [Figs. 7, 9]): 2^28
+    int32 as G = 2^28/N problems of N = 2^n, EVERY problem split into W contiguous portions
+    (portion r on rank r); one elements-mode call per step with G totals per rank exchanged
+    (fused peer stores; NCCL all-gather beside it).  Strong scaling (the 2^28 total is fixed).
+    At W = 1 the same pipeline runs with no peer, and the AUTO single-GPU scan of the same
+    batch is reported beside it."""
+    import inputs
+    from paper_conf_ipps_dieguezadnm18_b200 import multi
+    out = {}
+    hbm, _, _ = _peaks()
+    for n in logs:
+        N = 1 << n
+        G = (1 << 28) // N
+        a, b = multi.partition(N, world, rank)
+        L = b - a
+        x = torch.empty(G * L, dtype=torch.int32, device=dev)
+        inputs.fill_device(x, "i32", SEED + 20 + n, offset=a, row_len=0)
+        x = x.view(G, L)
+        y = torch.empty_like(x)
+        comms = _peer_comms(world, G)
+        times = {}
+        for name, c in comms.items():
+            times[name] = _time_calls(lambda: multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
+                                                               backend="peer" if name == "peer" else "native",
+                                                               comm=c), reps, world)
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        for c in comms.values():
+            c.close()
+        ms = times["peer"]
+        row = {"n": n, "N": N, "G": G, "N_per_gpu": L, "ms": ms, "Gelem/s": (1 << 28) / ms / 1e6,
+               "per_gpu_frac_measured_hbm_at_12B": 12.0 * G * L / (ms * 1e-3) / 1e9 / hbm,
+               "ms_by_exchange": times}
+        if world == 1:
+            sp = _time_alone(lambda: sb.scan(x, "add", "inclusive", out=y), reps)
+            row["single_gpu_auto_ms"] = sp
+            row["single_gpu_auto_kernel"] = "%s %s" % sb.plan(x, y)
+            row["single_gpu_auto_Gelem/s"] = (1 << 28) / sp / 1e6
+        out["n=%d" % n] = row
+        del x, y
+        torch.cuda.empty_cache()
+    return {"scaling": "strong (2^28 int32 per step, every problem split over the W ranks)",
+            "inputs": "synthetic int32 (splitmix64), each rank's own stream",
+            "points": out}
+
+
+# ---------------------------------------------------------------- configs[0] and configs[2]
+def device_time(fn, s, reps):
+    """Device time per call: warm up on stream s, capture `reps` calls into a CUDA graph,
+    replay it between two events (removes the Python/launch overhead from small cases)."""
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            fn()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(reps):
+            fn()
+    with torch.cuda.stream(s):
+        g.replay()
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(s)
+        g.replay()
+        s1.record(s)
+    torch.cuda.synchronize()
+    return s0.elapsed_time(s1) / reps
+
+
+def c1_latency(sb, dev, reps=50):
+    """configs[0]: N = 2^20, G = 1, inclusive int32 add: latency bound (8 MiB, L2-resident).
+    Reported warm (calls replayed back to back from a CUDA graph) and with L2 FLUSHED
+    (a 2 x L2 scratch buffer written between calls; events around each call only)."""
+    import inputs
+    x = torch.empty(1 << 20, dtype=torch.int32, device=dev)
+    inputs.fill_device(x, "i32", SEED + 1)
+    y = torch.empty_like(x)
+    gs = torch.cuda.Stream(dev)
+    warm_us = device_time(lambda: sb.scan(x, "add", out=y, stream=gs), gs, reps) * 1e3
+    flush = torch.empty(2 * 126 * (1 << 20) // 4, dtype=torch.int32, device=dev)
+    ts = []
+    for i in range(reps + 3):
+        flush.fill_(i)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        sb.scan(x, "add", out=y)
+        e1.record()
+        torch.cuda.synchronize()
+        if i >= 3:
+            ts.append(e0.elapsed_time(e1) * 1e3)
+    del flush
+    torch.cuda.empty_cache()
+    return {"us_per_scan_warm": warm_us, "Gelem/s_warm": (1 << 20) / warm_us / 1e3,
+            "us_per_scan_l2_flushed_median": statistics.median(ts), "us_per_scan_l2_flushed_min": min(ts),
+            "kernel": "%s %s" % sb.plan(x, y),
+            "note": "latency bound, no roofline claimed (8 MiB); warm = CUDA-graph replay of back-to-back "
+                    "calls; flushed = 252 MiB scratch written before each call, events around the call"}
+
+
+def roofline_c3(sb, dev, budget_cpu_s: float = 10.0, reps=10, with_cpu=True):
+    """configs[2]: one f32 add-scan of N = 2^30 (the L2-staged decoupled look-back), the
+    north_star's ">= 80 % of HBM for N >= 2^28" point, as its own roofline line: algorithmic
+    bytes 2 x 4 B x N per launch / the launch's device time (CUDA events around `reps`
+    back-to-back launches on the launching stream), against the measured copy bandwidth and
+    against the nominal 8 TB/s; ncu traffic from the hash-checked capture; the oracle timed
+    on the host on a bounded sample of the same input (streamed, fp64)."""
+    import inputs
+    N = 1 << 30
+    xi = torch.empty(N, dtype=torch.int32, device=dev)
+    inputs.fill_device(xi, "f32u", SEED + 3)
+    x = xi.view(torch.float32)
+    y = torch.empty_like(x)
+    for _ in range(3):
+        sb.scan(x, "add", out=y)
+    torch.cuda.synchronize()
+    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    for _ in range(reps):
+        sb.scan(x, "add", out=y)
+    s1.record()
+    torch.cuda.synchronize()
+    ms = s0.elapsed_time(s1) / reps
+    hbm, hbm_src, _ = _peaks()
+    bytes_launch = 8.0 * N
+    gbs = bytes_launch / (ms * 1e-3) / 1e9
+    algo, param = sb.plan(x, y)
+    traffic, tsrc = traffic_for("c3")
+    res = {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
+           "frac_of_nominal_8TBs": gbs / NOMINAL_HBM_GBS, "traffic": traffic, "traffic_src": tsrc,
+           "kernel": "%s [algo=%s param=%d] on f32 add inclusive, G=1 N=2^30" % (sb.KERNEL_NAMES[algo], algo, param),
+           "bytes_per_launch": bytes_launch, "ms_per_launch": ms, "Gelem/s": N / ms / 1e6,
+           "timing": "%d back-to-back launches between CUDA events on the launching stream" % reps,
+           "peak_src": hbm_src + " copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"}
+    if with_cpu:
+        # bounded sample: the streaming oracle over the first chunks of the SAME input (and a
+        # check of those output chunks, after timing)
+        import oracle
+        so = oracle.StreamAdd(np.float32, "inclusive")
+        step = 1 << 25
+        done, t_or, worst, ok = 0, 0.0, 0.0, True
+        while t_or < budget_cpu_s and done < N:
+            xc = xi[done: done + step].cpu().numpy().view(np.float32)
+            t0 = time.perf_counter()
+            ref, sabs = so.feed(xc)
+            t_or += time.perf_counter() - t0
+            got = y[done: done + step].cpu().numpy()
+            err = np.abs(got.astype(np.float64) - ref)
+            ok = ok and bool(np.all(err <= 1e-5 * sabs))
+            worst = max(worst, float(np.max(err / np.maximum(sabs, 1e-300))))
+            done += xc.shape[0]
+        res["cpu_baseline"] = {"value": done / t_or / 1e9, "unit": "Gelem/s", "cores": 1, "kind": "oracle",
+                               "sample": "first %d of the 2^30 elements of the c3 input, streamed f32->fp64 "
+                                         "sequential oracle (oracle_stream_add_f32), %.1f s" % (done, t_or),
+                               "host_cpu": _cpu_name()}
+        res["validated"] = {"elements": done, "ok": ok, "worst_err_over_sum_abs": worst}
+    del xi, x, y
+    torch.cuda.empty_cache()
+    return res
+
+
 # ---------------------------------------------------------------- CPU oracle (reference arm / baseline)
 def cpu_oracle_rate(budget_s: float = 12.0):
     """The oracle as it stands (one thread, sequential C loop) on the same workload: it
@@ -340,124 +709,6 @@ def _cpu_name():
     return "unknown"
 
 
-# ---------------------------------------------------------------- extra configs (context)
-def extras(sb, dev):
-    import inputs
-    out = {}
-    # c1: N = 2^20, G = 1, inclusive int32 add: latency-bound, L2 resident
-    x = torch.empty(1 << 20, dtype=torch.int32, device=dev)
-    inputs.fill_device(x, "i32", SEED + 1)
-    y = torch.empty_like(x)
-    for _ in range(10):
-        sb.scan(x, "add", out=y)
-    s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    torch.cuda.synchronize()
-    s0.record()
-    for _ in range(200):
-        sb.scan(x, "add", out=y)
-    s1.record()
-    torch.cuda.synchronize()
-    us = s0.elapsed_time(s1) / 200 * 1e3
-    gs = torch.cuda.Stream(dev)
-    dev_us = device_time(lambda: sb.scan(x, "add", out=y, stream=gs), gs, 50) * 1e3
-    out["c1_i32_incl_N2^20"] = {"us_per_scan_device": dev_us, "Gelem/s_device": (1 << 20) / dev_us / 1e3,
-                                "us_per_scan_host_launch": us,
-                                "note": "L2-resident (8 MiB); device = 50 launches replayed from a CUDA graph; "
-                                        "host_launch = back-to-back Python calls (host-bound)",
-                                "kernel": "%s %s" % sb.plan(x, y)}
-    del x, y
-    # c3: N = 2^30 f32 inclusive add, single problem (look-back)
-    N = 1 << 30
-    x = torch.empty(N, dtype=torch.int32, device=dev)
-    inputs.fill_device(x, "f32u", SEED + 3)
-    x = x.view(torch.float32)
-    y = torch.empty_like(x)
-    for _ in range(3):
-        sb.scan(x, "add", out=y)
-    torch.cuda.synchronize()
-    s0.record()
-    for _ in range(10):
-        sb.scan(x, "add", out=y)
-    s1.record()
-    torch.cuda.synchronize()
-    ms = s0.elapsed_time(s1) / 10
-    hbm, _, _ = _peaks()
-    gbs = 8.0 * N / (ms * 1e-3) / 1e9
-    out["c3_f32_incl_N2^30"] = {"ms": ms, "Gelem/s": N / ms / 1e6, "GB/s": gbs,
-                                "frac_measured_hbm": gbs / hbm, "frac_8TBs": gbs / 8000.0}
-    del x, y
-    torch.cuda.empty_cache()
-    return out
-
-
-def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB200_BENCH_ELEMS_LOG2", "33")),
-                  reps=10):
-    """configs[4]: one int32 add-scan sharded by elements (Multi-GPU Problem Scattering,
-    PAPER.md:195-205): each rank owns a contiguous 2^33-element portion (32 GiB in + 32 GiB
-    out) of ONE problem -- at W = 8 the problem is configs[4]'s N = 2^36.  Stage 1+2 ->
-    exchange -> Stage 3.  Weak-scaled (N = W x 2^33).  At W = 1 the same two-pass pipeline
-    runs with no peer (its 1-GPU reference rate)."""
-    import inputs
-    from paper_conf_ipps_dieguezadnm18_b200 import multi
-    x = torch.empty(n_local, dtype=torch.int32, device=dev)
-    inputs.fill_device(x, "i32", SEED + 5, offset=rank * n_local)
-    y = torch.empty_like(x)
-    # the fused exchange (Stage 2 pushes the totals into later ranks' HBM, Stage 3 waits on
-    # the device; no collective call) is the product path; NCCL all-gather beside it
-    comms = {"peer": multi.PeerComm(1) if world > 1 else multi.PeerComm.loopback(1, 1)[0]}
-    if world > 1 and DIST_BACKEND == "nccl":
-        comms["nccl"] = multi.NativeComm()
-
-    def run(name):
-        multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
-                         backend="peer" if name == "peer" else "native", comm=comms[name])
-    times = {}
-    for name in comms:
-        for _ in range(3):
-            run(name)
-        torch.cuda.synchronize()
-        if world > 1:
-            torch.distributed.barrier()
-        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s0.record()
-        for _ in range(reps):
-            run(name)
-        s1.record()
-        torch.cuda.synchronize()
-        times[name] = max_over_ranks(s0.elapsed_time(s1) / reps, world)
-    torch.cuda.synchronize()
-    if world > 1:
-        torch.distributed.barrier()
-    for c in comms.values():
-        c.close()
-    ms = times["peer"]
-    # per-phase breakdown (the paper's Fig. 14, PAPER.md:283-289): Stage 1+2 / exchange /
-    # Stage 3, events between the three steps of the torch-backend path
-    ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
-    ph = [0.0, 0.0, 0.0]
-    t = sb.shard_totals(x, "add")                 # warm-up (workspace growth), totals reused
-    torch.cuda.synchronize()
-    for _ in range(reps):
-        ev[0].record()
-        sb.shard_totals(x, "add", totals=t)
-        ev[1].record()
-        allt = all_gather_totals(t, world)
-        ev[2].record()
-        sb.shard_scan(x, allt, rank, world, "add", "inclusive", out=y)
-        ev[3].record()
-        torch.cuda.synchronize()
-        for k in range(3):
-            ph[k] += ev[k].elapsed_time(ev[k + 1]) / reps
-    hbm, _, _ = _peaks()
-    per_gpu_gbs = 12.0 * n_local / (ms * 1e-3) / 1e9          # reduce pass (4 B) + scan pass (8 B)
-    return {"N_total": world * n_local, "N_per_gpu": n_local, "ms": ms,
-            "Gelem/s": world * n_local / ms / 1e6, "per_gpu_GB/s_at_12B_per_elem": per_gpu_gbs,
-            "per_gpu_frac_measured_hbm": per_gpu_gbs / hbm,
-            "exchange": ("fused peer stores in the Stage 2/3 kernels (scan_comm_create_peer)" if world > 1
-                         else "none (W=1; the fused-exchange kernels run with no peers)"),
-            "ms_by_exchange": times,
-            "phases_ms_rank%d" % rank: {"stage1+2_reduce": ph[0], "exchange": ph[1], "stage3_scan": ph[2]}}
-
 
 def sweep(sb, dev):
     """On-box parameter search (the automated form of the paper's K search)."""
@@ -490,28 +741,37 @@ def sweep(sb, dev):
     return rows
 
 
-def device_time(fn, s, reps):
-    """Device time per call: warm up on stream s, capture `reps` calls into a CUDA graph,
-    replay it between two events (removes the Python/launch overhead from small cases)."""
-    with torch.cuda.stream(s):
-        for _ in range(3):
-            fn()
-    torch.cuda.synchronize()
-    g = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(g, stream=s):
-        for _ in range(reps):
-            fn()
-    with torch.cuda.stream(s):
-        g.replay()
-        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s0.record(s)
-        g.replay()
-        s1.record(s)
-    torch.cuda.synchronize()
-    return s0.elapsed_time(s1) / reps
-
-
 # ---------------------------------------------------------------- main
+def _config(world):
+    return {"workload": "configs[1]: batch scan G=4096 x N=2^14 per GPU, int32 and f32 add, "
+                        "inclusive and exclusive (4 scans per step)",
+            "G_per_gpu": G_C2, "N": N_C2, "layout": "row-major, stride N",
+            "l2": "inputs larger than L2 (256 MiB in + 256 MiB out per scan), no flush",
+            "parallelism": ("problems sharded by rank (Case 1), dp%d" % world) if world > 1 else "single GPU"}
+
+
+def dry_run(args, world, rank):
+    """Rank plumbing only (no GPU): gloo group, barrier, max over ranks, rank 0 prints."""
+    if world > 1:
+        torch.distributed.init_process_group("gloo")
+    global DIST_BACKEND
+    DIST_BACKEND = "gloo"
+    t0 = time.perf_counter()
+    if world > 1:
+        torch.distributed.barrier()
+    mine = float(rank + 1)
+    top = max_over_ranks(mine, world)
+    low = reduce_over_ranks(mine, world, "min")
+    wall = max_over_ranks((time.perf_counter() - t0) * 1e3, world)
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "value": None, "unit": "Gelem/s", "n_gpus": world,
+                          "steps": args.steps, "warmup": args.warmup, "dry_run": True,
+                          "ranks_seen": {"max": top, "min": low}, "plumbing_wall_ms": wall,
+                          "config": _config(world)}), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -521,18 +781,18 @@ def main():
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", action="store_true")
-    ap.add_argument("--no-cpu", action="store_true", help="skip the CPU oracle baseline (profiling runs)")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the CPU oracle baselines (profiling runs)")
+    ap.add_argument("--dry-run", action="store_true", help="rank plumbing only, no GPU (CPU hosts)")
     args = ap.parse_args()
+    maybe_respawn(args)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.dry_run:
+        return dry_run(args, world, rank)
     hbm, hbm_src, _ = _peaks()
-    config = {"workload": "configs[1]: batch scan G=4096 x N=2^14 per GPU, int32 and f32 add, "
-                          "inclusive and exclusive (4 scans per step)",
-              "G_per_gpu": G_C2, "N": N_C2, "layout": "row-major, stride N",
-              "l2": "inputs larger than L2 (256 MiB in + 256 MiB out per scan), no flush",
-              "parallelism": "problems sharded by rank (Case 1)" if world > 1 else "single GPU"}
+    config = _config(world)
 
     if args.impl == "reference":
         if rank != 0:
@@ -570,14 +830,16 @@ def main():
         step(sb, xs, outs)
     torch.cuda.synchronize()
 
-    # timed region: barrier + synchronize on both sides, device events, max over ranks
-    if world > 1:
-        torch.distributed.barrier()
+    # timed region: barrier + aligning all-reduce + synchronize on both sides, device events,
+    # max over ranks; the host wall clock of the same region beside it (cross-check)
     with ClockSampler(local) as clk:
-        total_ms, _ = timed_steps(sb, xs, outs, args.steps)
+        total_ms, wall_ms = timed_steps(sb, xs, outs, args.steps, world)
     if world > 1:
         torch.distributed.barrier()
-        total_ms = max_over_ranks(total_ms, world)
+    total_ms = max_over_ranks(total_ms, world)
+    wall_ms = max_over_ranks(wall_ms, world)
+    validation = validate_step(xs, outs)
+    ok_all = max_over_ranks(0.0 if validation["ok"] else 1.0, world) == 0.0
     # average launch duration of the dominant kernel, live over the timed region: every
     # launch in it is the same kernel family on the same bytes (the plan is checked below),
     # so it is the timed region's device time / its launches.  Events between launches are
@@ -585,7 +847,7 @@ def main():
     # Per-variant averages (reps back-to-back launches of one call between two events on the
     # launching stream) are reported beside it.
     launch_ms = kernel_times(sb, xs, outs, max(20, args.steps // 4))
-    plans = {sb.plan(xs[dt], outs[i]) for i, (dt, _, _) in enumerate(VARIANTS)}
+    plans = {sb.plan(xs[dt], outs[i], op=op, kind=kind) for i, (dt, op, kind) in enumerate(VARIANTS)}
     live_launch_ms = total_ms / (args.steps * len(VARIANTS))
 
     ms_step = total_ms / args.steps
@@ -599,14 +861,8 @@ def main():
     else:
         achieved, dom_ms, timing = (bytes_launch / (launch_ms[dom] * 1e-3) / 1e9, launch_ms[dom],
                                     "back-to-back launches of the slowest variant between two events")
-    algo, param = sb.plan(xs[VARIANTS[dom][0]], outs[dom])
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tpath):
-        try:
-            traffic = json.load(open(tpath)).get("bytes_per_launch")
-        except Exception:
-            traffic = None
+    algo, param = sb.plan(xs[VARIANTS[dom][0]], outs[dom], op=VARIANTS[dom][1], kind=VARIANTS[dom][2])
+    traffic, tsrc = traffic_for("c2")
     res = {
         "metric": METRIC, "value": value, "unit": "Gelem/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
@@ -615,30 +871,40 @@ def main():
         "hbm_frac_of_step": {"algorithmic_GB/s": elems_step / world * 8 / (ms_step * 1e-3) / 1e9,
                              "frac": elems_step / world * 8 / (ms_step * 1e-3) / 1e9 / hbm, "peak_src": hbm_src},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved / hbm, "traffic": traffic,
+                     "frac": achieved / hbm, "frac_of_nominal_8TBs": achieved / NOMINAL_HBM_GBS,
+                     "traffic": traffic, "traffic_src": tsrc,
                      "kernel": "%s [algo=%s param=%d] on %s %s %s" % (
                          sb.KERNEL_NAMES[algo], algo, param, *VARIANTS[dom]),
                      "bytes_per_launch": bytes_launch, "ms_per_launch": dom_ms, "timing": timing,
                      "bytes_basis": "2 x 4 B x G x N (read input once, write output once)",
                      "peak_src": hbm_src + " copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"},
         "per_launch_ms": {"%s_%s_%s" % v: m for v, m in zip(VARIANTS, launch_ms)},
-
+        "wall_clock_check": {"wall_ms_per_step_max_over_ranks": wall_ms / args.steps,
+                             "device_over_wall": total_ms / wall_ms,
+                             "note": "host perf_counter around the same timed region (after the aligning "
+                                     "barrier, synchronize at the end); device time must not exceed it"},
+        "validation": validation,
         "gpu_launches": len(VARIANTS) * args.steps,
         "clocks": clk.summary(),
     }
+    if not ok_all:
+        if rank == 0:
+            res["error"] = "output validation failed on at least one rank"
+            print(json.dumps(res), flush=True)
+        raise SystemExit(3)
+    del xs, outs
+    torch.cuda.empty_cache()
     if not args.no_extras:
-        el = elements_mode(sb, dev, world, rank)
-        res["elements_mode_sharded_problem"] = el
-        torch.cuda.empty_cache()
+        res["elements_mode_sharded_problem"] = elements_mode(sb, dev, world, rank)
+        res["scan_mps"] = scan_mps(sb, dev, world, rank)
         res["c4_problems_mode"] = c4_problems(sb, dev, world, rank)
     if not args.no_e2e:
         res["e2e"] = e2e(sb, world)
     if rank == 0 and world == 1 and not args.no_cpu:
         res["cpu_baseline"] = cpu_oracle_rate()
     if rank == 0 and world == 1 and not args.no_extras:
-        del xs, outs
-        torch.cuda.empty_cache()
-        res["extras"] = extras(sb, dev)
+        res["roofline_c3"] = roofline_c3(sb, dev, with_cpu=not args.no_cpu)
+        res["extras"] = {"c1_i32_incl_N2^20": c1_latency(sb, dev)}
     if rank == 0:
         print(json.dumps(res), flush=True)
     if world > 1:
