@@ -223,6 +223,12 @@ scan_status resolve_ws(void* ws, size_t ws_bytes, size_t need, cudaStream_t s, i
 // it, for A/B measurements)
 const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
 
+// look-back polling / tail options (A/B switches for on-box measurements)
+const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 4;
+const bool g_keep_last = std::getenv("SCANB200_NO_KEEP_LAST") == nullptr;
+const int g_lb_tail = std::getenv("SCANB200_LB_TAIL") ? std::atoi(std::getenv("SCANB200_LB_TAIL")) : 1;
+const uint32_t g_poll_ns = (uint32_t)std::atoi(std::getenv("SCANB200_POLL_NS") ? std::getenv("SCANB200_POLL_NS") : "64");
+
 // debug timeline buffer for the look-back kernels (scan_debug_trace)
 uint64_t* g_trace = nullptr;
 int64_t g_trace_tiles = 0;
@@ -268,6 +274,10 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
     p.exclusive = kind == SCAN_EXCLUSIVE;
     p.pdl_first = g_cross_pdl;
+    p.lb_mode = g_lb_mode;
+    p.keep_last = g_keep_last;
+    p.poll_ns = g_poll_ns;
+    p.lb_tail = g_lb_tail;
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
 }
 

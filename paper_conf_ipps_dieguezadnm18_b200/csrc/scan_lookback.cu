@@ -84,6 +84,25 @@ struct Desc {
             st_relaxed_u64(p.desc + kDescWords * t, ((uint64_t)to_bits<C>(v) << 32) | meta);
         }
     }
+    // raw load of a slot (issued without consuming the result, so a warp can have every
+    // load of a window in flight at once) and its decoding
+    struct Raw { uint64_t a, b; };
+    static __device__ __forceinline__ void load(const LookbackParams& p, int64_t t, Raw& r) {
+        if constexpr (sizeof(C) == 8) ld_relaxed_v2u64(p.desc + kDescWords * t, r.a, r.b);
+        else r.a = ld_relaxed_u64(p.desc + kDescWords * t);
+    }
+    static __device__ __forceinline__ uint32_t decode(const Raw& r, uint32_t tag, C& v) {
+        if constexpr (sizeof(C) == 8) {
+            const uint32_t mh = (uint32_t)r.a, ml = (uint32_t)r.b;
+            if ((mh >> 2) != tag || mh != ml) return 0u;
+            v = __longlong_as_double((long long)((r.a & 0xFFFFFFFF00000000ull) | (r.b >> 32)));
+            return mh & 3u;
+        } else {
+            if ((((uint32_t)r.a) >> 2) != tag) return 0u;
+            v = from_bits<C>((uint32_t)(r.a >> 32));
+            return (uint32_t)r.a & 3u;
+        }
+    }
     // returns status (0 when stale, torn or not yet written) and the matching value
     static __device__ __forceinline__ uint32_t read(const LookbackParams& p, int64_t t, uint32_t tag, C& v) {
         if constexpr (sizeof(C) == 8) {
@@ -153,6 +172,170 @@ __device__ __forceinline__ typename Op::Carry look_back(const LookbackParams& p,
     return run;
 }
 
+// The same look-back with the window's loads in flight together (one L2 round trip per
+// poll instead of M, the serialised form above) and re-polls that re-read only the
+// descriptors still missing before the nearest P, with an exponential back-off starting at
+// p.poll_ns -- so a waiting warp does not flood the descriptor lines the streaming traffic
+// shares L2 with.
+template <class Op, int M = LB_M>
+__device__ __forceinline__ typename Op::Carry look_back_par(const LookbackParams& p, int64_t t, uint32_t tag,
+                                                            uint32_t* stats = nullptr) {
+    using C = typename Op::Carry;
+    using Raw = typename Desc<Op>::Raw;
+    const int lane = lane_id();
+    C run = Op::cidentity();
+    int64_t front = t - 1;
+    while (true) {
+        C v[M];
+        uint32_t st[M];
+        Raw r[M];
+        if (stats) { stats[1] += 1; stats[0] += 1; }
+#pragma unroll
+        for (int m = 0; m < M; ++m) {
+            const int64_t pred = front - lane - 32 * m;
+            r[m].a = r[m].b = 0ull;
+            if (pred >= 0) Desc<Op>::load(p, pred, r[m]);
+        }
+#pragma unroll
+        for (int m = 0; m < M; ++m) {
+            const int64_t pred = front - lane - 32 * m;
+            v[m] = Op::cidentity();
+            st[m] = pred >= 0 ? Desc<Op>::decode(r[m], tag, v[m]) : ST_P;
+        }
+        int dP;
+        uint32_t ns = p.poll_ns;
+        while (true) {
+            dP = 1 << 30;
+#pragma unroll
+            for (int m = M - 1; m >= 0; --m) {
+                const unsigned pm = __ballot_sync(FULL, st[m] == ST_P);
+                if (pm) dP = 32 * m + __ffs(pm) - 1;
+            }
+            bool pend[M];
+            bool any = false;
+#pragma unroll
+            for (int m = 0; m < M; ++m) {
+                pend[m] = st[m] == 0u && (lane + 32 * m) < dP;
+                any = any || (__ballot_sync(FULL, pend[m]) != 0u);
+            }
+            if (!any) break;
+            if (ns) { __nanosleep(ns); if (ns < 2048u) ns <<= 1; }
+            if (stats) stats[0] += 1;
+#pragma unroll
+            for (int m = 0; m < M; ++m)
+                if (pend[m]) Desc<Op>::load(p, front - lane - 32 * m, r[m]);
+#pragma unroll
+            for (int m = 0; m < M; ++m)
+                if (pend[m]) st[m] = Desc<Op>::decode(r[m], tag, v[m]);
+        }
+        C mine = Op::cidentity();
+#pragma unroll
+        for (int m = 0; m < M; ++m)
+            if (lane + 32 * m <= dP && front - lane - 32 * m >= 0) mine = Op::capply(v[m], mine);
+        run = Op::capply(warp_reduce_carry<Op>(mine), run);   // the window is older than `run`
+        if (dP < (1 << 30)) break;
+        front -= 32 * M;
+    }
+    return run;
+}
+
+// Look-back of a PERSISTENT round-robin grid (tile t = cta + i * grid): the CTA's own
+// previous tile t - grid was resolved by this CTA, so its inclusive prefix is known in
+// shared memory (s_incl, tagged with its sequence number in s_iseq).  The carry of t is
+//     incl(t - grid)  .  A(t - grid + 1)  .  ...  .  A(t - 1)
+// or, if one of those window tiles already published its inclusive value P, the fold from
+// the nearest P.  So the window never slides past t - grid: one window of grid - 1 <= 32 M
+// descriptors, loaded together; re-polls re-read only the descriptors still missing (X),
+// with back-off; once every window tile has at least its aggregate the warp waits on
+// shared memory only (no L2 traffic).  If the local slot was already lapped (the ring holds
+// 2 x SH sequences), tile t - grid's P descriptor is read instead (it was published before
+// the slot was written).
+template <class Op, int M>
+__device__ __forceinline__ typename Op::Carry look_back_rr(const LookbackParams& p, int64_t t, int64_t i, int64_t grid,
+                                                           uint32_t tag, const typename Op::Carry* s_incl,
+                                                           const int64_t* s_iseq, int ring, uint32_t* stats) {
+    using C = typename Op::Carry;
+    using Raw = typename Desc<Op>::Raw;
+    const int lane = lane_id();
+    const int64_t span = grid - 1;
+    C v[M];
+    uint32_t st[M];
+    Raw r[M];
+    if (stats) { stats[1] += 1; stats[0] += 1; }
+#pragma unroll
+    for (int m = 0; m < M; ++m) {
+        const int64_t d = 1 + lane + 32 * m;
+        r[m].a = r[m].b = 0ull;
+        if (d <= span) Desc<Op>::load(p, t - d, r[m]);
+    }
+#pragma unroll
+    for (int m = 0; m < M; ++m) {
+        const int64_t d = 1 + lane + 32 * m;
+        v[m] = Op::cidentity();
+        st[m] = d <= span ? Desc<Op>::decode(r[m], tag, v[m]) : ST_A;     // outside: identity
+    }
+    const int slot = (int)((i - 1) % ring);
+    bool have_local = false;
+    C local = Op::cidentity();
+    int dP;
+    uint32_t ns = p.poll_ns;
+    while (true) {
+        dP = 1 << 30;
+#pragma unroll
+        for (int m = M - 1; m >= 0; --m) {
+            const unsigned pm = __ballot_sync(FULL, st[m] == ST_P);
+            if (pm) dP = 32 * m + __ffs(pm) - 1;
+        }
+        bool pend[M];
+        bool any = false;
+#pragma unroll
+        for (int m = 0; m < M; ++m) {
+            pend[m] = st[m] == 0u && (lane + 32 * m) < dP;
+            any = any || (__ballot_sync(FULL, pend[m]) != 0u);
+        }
+        if (!any) {
+            if (dP < (1 << 30)) break;                   // fold from the nearest P
+            const int64_t q = *(const volatile int64_t*)(s_iseq + slot);
+            if (q == i - 1) {
+                __threadfence_block();
+                local = *(const volatile C*)(s_incl + slot);
+                have_local = true;
+                break;
+            }
+            if (q > i - 1) {                             // lapped: tile t - grid's P is global
+                C pv = Op::cidentity();
+                while (Desc<Op>::read(p, t - grid, tag, pv) != ST_P) __nanosleep(64);
+                local = pv;
+                have_local = true;
+                break;
+            }
+            __nanosleep(20);                             // local prefix not ready: smem only
+            continue;
+        }
+        if (ns) { __nanosleep(ns); if (ns < 2048u) ns <<= 1; }
+        if (stats) stats[0] += 1;
+#pragma unroll
+        for (int m = 0; m < M; ++m)
+            if (pend[m]) Desc<Op>::load(p, t - 1 - lane - 32 * m, r[m]);
+#pragma unroll
+        for (int m = 0; m < M; ++m)
+            if (pend[m]) st[m] = Desc<Op>::decode(r[m], tag, v[m]);
+    }
+    C mine = Op::cidentity();
+#pragma unroll
+    for (int m = 0; m < M; ++m)
+        if (lane + 32 * m <= dP) mine = Op::capply(v[m], mine);
+    C run = warp_reduce_carry<Op>(mine);
+    if (have_local) run = Op::capply(local, run);
+    return run;
+}
+
+template <class Op, int M = LB_M>
+__device__ __forceinline__ typename Op::Carry look_back_any(const LookbackParams& p, int64_t t, uint32_t tag,
+                                                            uint32_t* stats = nullptr) {
+    return p.lb_mode == 1 ? look_back_par<Op, M>(p, t, tag, stats) : look_back<Op, M>(p, t, tag, stats);
+}
+
 // debug timeline (scan_debug_trace): stamp e of tile t with %globaltimer (ns)
 __device__ __forceinline__ void trace_stamp(const LookbackParams& p, int64_t t, int e) {
     if (p.trace != nullptr && t < p.trace_tiles) {
@@ -209,7 +392,7 @@ __device__ __forceinline__ void tile_body_smem(const LookbackParams& p, int64_t 
         const C aggc = Op::to_carry(agg);
         if (lane == 0) Desc<Op>::publish(p, tile, tag, has_head ? ST_P : ST_A, aggc);
         C carry = Op::cidentity();
-        if (!starts) carry = look_back<Op>(p, tile, tag);
+        if (!starts) carry = look_back_any<Op>(p, tile, tag);
         if (lane == 0) {
             if (!has_head) Desc<Op>::publish(p, tile, tag, ST_P, Op::capply(carry, aggc));
             *s_carry = carry;
@@ -271,6 +454,7 @@ struct SlotHdr {
     int64_t tid;
     int64_t r;
     uint32_t seg, fast;
+    uint32_t keep;          // L2-staged kernel: scan this tile from its read-1 slot
     T wtot[WARPS];
     uint32_t wfl[WARPS];
     T wp[WARPS];
@@ -482,7 +666,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
             if (lane == 0) trace_stamp(p, t, 4);
-            if (!starts) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            if (!starts) carry = look_back_any<Op, M>(p, t, tag, p.trace ? stats : nullptr);
             mbar_wait(&s_p1[slot], ph);                   // this tile's aggregate is in the header
             SlotHdr<Op, WARPS>& h = s_hdr[slot];
             const bool has_head = h.has_head != 0u;
@@ -535,6 +719,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int V = 8, WCH = V * 128, TILE = NS * WCH;
+    static_assert(SR >= 2, "a kept last tile must leave a read-1 slot for the end sentinel");
     extern __shared__ __align__(128) unsigned char dsm[];
     T* bufR = (T*)dsm;                       // SR x TILE
     T* bufW = bufR + (size_t)SR * TILE;      // SW x TILE
@@ -542,6 +727,9 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     __shared__ uint64_t fullR[SR], emptyR[SR], fullW[SW], emptyW[SW], aggd[SH], crd[SH], emptyH[SH];
     __shared__ uint32_t s_tag;
     __shared__ int64_t s_end;
+    constexpr int RING = 2 * SH;             // local inclusive prefixes of this CTA's tiles
+    __shared__ C s_incl[RING];
+    __shared__ int64_t s_iseq[RING];
     const int warp = threadIdx.x >> 5, lane = lane_id();
     // every CTA is resident before a dependent grid can launch (launch_dependents counts
     // all of them), so the static round robin's inter-CTA waits cannot be starved of SMs;
@@ -554,6 +742,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         for (int s = 0; s < SR; ++s) { mbar_init(&fullR[s], 1); mbar_init(&emptyR[s], NR); }
         for (int s = 0; s < SW; ++s) { mbar_init(&fullW[s], 1); mbar_init(&emptyW[s], NS); }
         for (int s = 0; s < SH; ++s) { mbar_init(&aggd[s], 1); mbar_init(&crd[s], 1); mbar_init(&emptyH[s], NS); }
+        for (int s = 0; s < RING; ++s) s_iseq[s] = -1;
         fence_mbar_init();
         s_tag = read_tag(p);
     }
@@ -569,7 +758,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const SlotHdr<Op, NS>& h = s_hdr[sH];
             const int64_t t = h.tid;
             if (t < 0) break;
-            const T* srow = bufW + (size_t)sW * TILE + warp * WCH;
+            // a kept tile (the CTA's last) is still in its read-1 slot: no second read
+            const T* srow = (h.keep ? bufR + (size_t)(i % SR) * TILE : bufW + (size_t)sW * TILE) + warp * WCH;
             const T cin = Op::from_carry(h.carry);
             const T wp = h.wp[warp];
             const bool wpf = h.wpf[warp] != 0u, fast = h.fast != 0u;
@@ -625,7 +815,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                 if (lane == 0) { h.wtot[k] = tot; h.wfl[k] = fl ? 1u : 0u; }
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&emptyR[sR]);
+            // a kept tile keeps its slot (read-1 never reuses it: the CTA has no later tile)
+            if (lane == 0 && !h.keep) mbar_arrive(&emptyR[sR]);
             asm volatile("bar.sync 2, %0;" :: "r"(NR * 32) : "memory");
             if (rr == NR - 1) {
                 T run = Op::identity(); bool f = false;
@@ -664,7 +855,10 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const TileInfo ti = classify(p, t, TILE);
             T* dst = bufR + (size_t)sR * TILE;
             const int64_t base = t * (int64_t)TILE;
-            if (lane == 0) { h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast; }
+            if (lane == 0) {
+                h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast;
+                h.keep = (p.keep_last && t + (int64_t)gridDim.x >= num_tiles) ? 1u : 0u;
+            }
             if (ti.fast) {
                 if (lane == 0) {
                     mbar_expect_tx(&fullR[sR], TILE * 4);
@@ -696,7 +890,9 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             }
             T* dst = bufW + (size_t)sW * TILE;
             const int64_t base = t * (int64_t)TILE;
-            if (h.fast) {
+            if (h.keep) {
+                if (lane == 0) mbar_arrive(&fullW[sW]);      // data already in the read-1 slot
+            } else if (h.fast) {
                 if (lane == 0) {
                     mbar_expect_tx(&fullW[sW], TILE * 4);
                     tma_load_1d(dst, in + base, TILE * 4, &fullW[sW], pol);
@@ -720,18 +916,45 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
+            // mode 4 (lazy): the look-back starts once this tile's own aggregate is out --
+            // its predecessors' aggregates arrive around the same time, so the window is
+            // (nearly) complete at the first poll and no warp spins on descriptors that
+            // cannot be ready yet (such polls slow the streaming reads they share L2 with)
+            const bool lazy = p.lb_mode == 4;
+            if (lazy) mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
             if (i < n_mine) {
                 if (lane == 0) trace_stamp(p, t, 4);
-                if (((t * (int64_t)TILE) % p.N) != 0) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+                if (((t * (int64_t)TILE) % p.N) != 0 && lazy) {
+                    if (i > 0 && (int64_t)gridDim.x - 1 <= 32 * M)
+                        carry = look_back_rr<Op, M>(p, t, i, gridDim.x, tag, s_incl, s_iseq, RING,
+                                                    p.trace ? stats : nullptr);
+                    else
+                        carry = look_back_par<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+                } else if (((t * (int64_t)TILE) % p.N) != 0) {
+                    // mode 3: the serial (self-throttling) poll while the CTA streams, the
+                    // round-robin window with loads in flight for its last lb_tail tiles
+                    // (the kernel's drain, when no streaming traffic competes any more)
+                    const bool rr = p.lb_mode == 2 || (p.lb_mode == 3 && i + p.lb_tail >= n_mine);
+                    if (rr && i > 0 && (int64_t)gridDim.x - 1 <= 32 * M)
+                        carry = look_back_rr<Op, M>(p, t, i, gridDim.x, tag, s_incl, s_iseq, RING,
+                                                    p.trace ? stats : nullptr);
+                    else
+                        carry = look_back_any<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+                }
             }
-            mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
+            if (!lazy) mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
             SlotHdr<Op, NS>& h = s_hdr[sH];
             if (i == n_mine) {                       // forward the end sentinel to P2
                 if (lane == 0) mbar_arrive(&crd[sH]);
                 break;
             }
             if (lane == 0) {
-                if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, Op::capply(carry, h.agg));
+                const C incl = h.has_head ? h.agg : Op::capply(carry, h.agg);
+                if (!h.has_head) Desc<Op>::publish(p, t, tag, ST_P, incl);
+                // the next tile of this CTA (another look-back warp) takes it from here
+                s_incl[i % RING] = incl;
+                __threadfence_block();
+                *(volatile int64_t*)(s_iseq + (i % RING)) = i;
                 h.carry = carry;
                 trace_stamp(p, t, 2);
                 trace_value(p, t, 5, stats[0]);
@@ -853,7 +1076,7 @@ __device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t ti
         if (lane == 0) { trace_stamp(p, tile, 1); trace_stamp(p, tile, 4); }
         C carry = Op::cidentity();
         uint32_t stats[2] = {0u, 0u};
-        if (!starts) carry = look_back<Op>(p, tile, tag, p.trace ? stats : nullptr);
+        if (!starts) carry = look_back_any<Op>(p, tile, tag, p.trace ? stats : nullptr);
         if (lane == 0) {
             if (!has_head) Desc<Op>::publish(p, tile, tag, ST_P, Op::capply(carry, aggc));
             trace_stamp(p, tile, 2);

@@ -40,8 +40,7 @@ def graph_ms(fn, reps):
     return best
 
 
-CANDS = [("auto", -1), ("lookback", 1), ("lookback", 2), ("lookback", 10), ("lookback", 11),
-         ("lookback", 12), ("lookback", 13), ("lookback", 14), ("cluster", -1), ("three_stage", 0), ("three_stage", 1), ("three_stage", 2), ("cascade_cta", -1)]
+CANDS = [("auto", -1), ("lookback", 1), ("lookback", 2), ("lookback", 3), ("lookback", 10), ("cluster", -1), ("three_stage", 0), ("three_stage", 1), ("three_stage", 2), ("cascade_cta", -1)]
 
 
 def main():

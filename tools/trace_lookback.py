@@ -19,6 +19,7 @@ ap.add_argument("--G", type=int, default=1)
 ap.add_argument("--N", type=int, default=1 << 28)
 ap.add_argument("--param", type=int, default=0)
 ap.add_argument("--tile", type=int, default=0, help="tile elements (default: from the variant)")
+ap.add_argument("--save", default="", help="save the raw [tiles, 8] trace as .npy")
 a = ap.parse_args()
 dt = {"i32": torch.int32, "f32": torch.float32}[a.dtype]
 x = torch.empty(a.G * a.N, dtype=torch.int32, device="cuda")
@@ -36,6 +37,8 @@ sb.scan(x, "add", out=y, algo="lookback", param=a.param)
 torch.cuda.synchronize()
 _lib.lib.scan_debug_trace(None, 0)
 R = tr.cpu().numpy().reshape(tiles, 8).astype(np.int64)
+if a.save:
+    np.save(a.save, R)
 T = R[:, :5].copy()
 T = T - T[:, 0].min()
 print("tiles", tiles, "span us %.1f" % (T[:, 3].max() / 1e3))
