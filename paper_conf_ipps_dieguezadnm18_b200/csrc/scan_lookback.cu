@@ -19,10 +19,13 @@
 //      persistent, one CTA per SM, tiles of 8192 elements (32 KiB) assigned round robin
 //      (tile = cta + k * grid, launched cooperatively so the whole grid is co-resident);
 //      every tile is read TWICE but from HBM once: read 1 (TMA bulk copy into a smem ring,
-//      SASS UBLKCP) feeds 4 reducer warps that publish the tile aggregate (A) at once and
-//      free the slot; 8 speculative look-back warps resolve the carry while the data waits
-//      in L2; read 2 (L2 -> smem) feeds 8 scanner warps that add the carry and store.
-//      The next round's read 1 is L2-prefetched (UBLKPF).  ~102 % of measured copy at 2^30.
+//      SASS UBLKCP) feeds 8 reducer warps that publish the tile aggregate (A) at once and
+//      free the slot; 2 look-back warps resolve the carry LAZILY (from the tile's own A
+//      on: the window of the grid - 1 predecessors is loaded in one round trip and the CTA's
+//      own previous tile supplies the inclusive prefix from shared memory) while the data
+//      waits in L2; read 2 (L2 -> smem) feeds 8 scanner warps that add the carry and store
+//      (the CTA's last tile is scanned from its read-1 slot).  The next round's read 1 is
+//      L2-prefetched (UBLKPF).  ~100 % of measured copy from 2^27 on, 0.82 / 0.90 at 2^24 / 2^25.
 //   0/1 lookback_pipelined_kernel -- persistent, one read: a producer warp streams 64 / 32
 //      KiB tiles into a 3-slot TMA ring, 16 / 8 consumer warps scan each staged tile in two
 //      passes, a dedicated look-back warp resolves the carry (window of 160 / 128 tiles);
@@ -417,8 +420,11 @@ __device__ __forceinline__ TileInfo classify(const LookbackParams& p, int64_t t,
 }
 
 // The last CTA to finish resets the counters and advances the epoch (wrap: clear all).
+// No fence before the count: the epoch only has to advance after every CTA READ it (at
+// its start, long before); a descriptor store of this launch still in flight carries this
+// launch's tag, which no later launch accepts, so the CTA need not wait for its stores
+// here (the next kernel is ordered after this grid's completion anyway).
 __device__ __forceinline__ void epilogue(const LookbackParams& p) {
-    __threadfence();
     const uint32_t prev = atomicAdd(p.ctl + 1, 1u);
     if (prev == gridDim.x - 1) {
         __threadfence();
@@ -719,13 +725,12 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int V = 8, WCH = V * 128, TILE = NS * WCH;
-    static_assert(SR >= 2, "a kept last tile must leave a read-1 slot for the end sentinel");
+    static_assert(SR >= 2, "kept tail tiles must leave a read-1 slot for the end sentinel");
     extern __shared__ __align__(128) unsigned char dsm[];
     T* bufR = (T*)dsm;                       // SR x TILE
     T* bufW = bufR + (size_t)SR * TILE;      // SW x TILE
     __shared__ SlotHdr<Op, NS> s_hdr[SH];
     __shared__ uint64_t fullR[SR], emptyR[SR], fullW[SW], emptyW[SW], aggd[SH], crd[SH], emptyH[SH];
-    __shared__ uint32_t s_tag;
     __shared__ int64_t s_end;
     constexpr int RING = 2 * SH;             // local inclusive prefixes of this CTA's tiles
     __shared__ C s_incl[RING];
@@ -744,10 +749,11 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         for (int s = 0; s < SH; ++s) { mbar_init(&aggd[s], 1); mbar_init(&crd[s], 1); mbar_init(&emptyH[s], NS); }
         for (int s = 0; s < RING; ++s) s_iseq[s] = -1;
         fence_mbar_init();
-        s_tag = read_tag(p);
     }
     __syncthreads();
-    const uint32_t tag = s_tag;
+    // the launch tag (an L2 round trip) is read only by the warps that publish or read
+    // descriptors, so the first read-1 bulk copies are not queued behind it
+    const uint32_t tag = ((warp >= NS && warp < NS + NR) || warp >= NS + NR + 2) ? read_tag(p) : 0u;
     const T* in = (const T*)p.in;
 
     if (warp < NS) {
@@ -815,7 +821,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                 if (lane == 0) { h.wtot[k] = tot; h.wfl[k] = fl ? 1u : 0u; }
             }
             __syncwarp();
-            // a kept tile keeps its slot (read-1 never reuses it: the CTA has no later tile)
+            // a kept tile keeps its slot: read-1 never reuses it (at most SR - 1 tiles of the
+            // CTA are kept, and the end sentinel takes the remaining slot)
             if (lane == 0 && !h.keep) mbar_arrive(&emptyR[sR]);
             asm volatile("bar.sync 2, %0;" :: "r"(NR * 32) : "memory");
             if (rr == NR - 1) {
@@ -857,7 +864,9 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const int64_t base = t * (int64_t)TILE;
             if (lane == 0) {
                 h.tid = t; h.r = ti.r; h.seg = ti.seg; h.fast = ti.fast;
-                h.keep = (p.keep_last && t + (int64_t)gridDim.x >= num_tiles) ? 1u : 0u;
+                // the CTA's last SR - 1 tiles are scanned from their read-1 slots (no second
+                // read on the kernel's tail); the slots they keep are never needed again
+                h.keep = (p.keep_last && t + (int64_t)(SR - 1) * gridDim.x >= num_tiles) ? 1u : 0u;
             }
             if (ti.fast) {
                 if (lane == 0) {
@@ -1147,7 +1156,10 @@ cudaError_t launch_op(const LookbackParams& p, int variant, cudaStream_t s) {
     case 0: return launch_pipelined<Op, 16, 8, 3, 5, 1, 1>(p, s);  // 64 KiB tiles, window 160, L2 prefetch +1 round
     case 1: return launch_pipelined<Op, 8, 8, 3, 4, 1, 0>(p, s);   // 32 KiB tiles (small, L2-resident totals)
     case 2: return launch_tma<Op, 8, 8>(p, s);                     // one 8192-element tile per CTA
-    case 3: return launch_l2<Op, 8, 4, 3, 3, 8, 5, 8>(p, s);       // two reads (L2-staged), 8-tile header ring, 8 look-back warps
+    // two reads (L2-staged), 8-tile header ring; 8 scanner, 8 reducer and 2 look-back warps
+    // (18 warps: 96 registers per thread; the lazy look-back needs few warps -- measured
+    // against 4 reducers + 8 look-back warps: 2^24 0.79 -> 0.82, 2^25 0.85 -> 0.90 of copy)
+    case 3: return launch_l2<Op, 8, 8, 3, 3, 8, 5, 2>(p, s);
     case 10: return launch_regtile<Op, 16, 4>(p, s);               // one 8192-element register tile per CTA
     default: return cudaErrorInvalidValue;
     }
