@@ -76,10 +76,11 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // (2^15 < N <= 2^16 at G = 1: the two-launch chain 3.6 us vs the cluster 3.9-4.0 us once
     //  both use programmatic launch, profiles/r01_g1_probe_cluster_boundary.jsonl)
     if (G <= 64 && N <= 32768) return SCAN_ALGO_CLUSTER;
-    // three-stage up to 2^23 elements: the second read of the input still hits L2, and
-    // the chain beats the L2-staged look-back's fill/drain there (2^23: 16.3 vs 19.6 us;
-    // from 2^24 the look-back wins, profiles/r01_mid_probe.jsonl)
-    if (G <= 64 && N * G <= (int64_t(1) << 23) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    // three-stage up to ~7 x 2^20 elements: the second read of the input still hits L2, and
+    // the chain beats the L2-staged look-back's fill/drain there (6 x 2^20: 12.9 vs 13.5 us);
+    // the lazy look-back wins from 2^23 (15.0 vs 15.6 us i32, 14.9 vs 15.4 us f32;
+    // profiles/r02_g1_boundary.jsonl)
+    if (G <= 64 && N * G <= (int64_t(7) << 20) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     // a few hundred to a few thousand problems of moderate length (scan_autotune over a
     // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA
     // beat the flat look-back 1.1-4.8x there (e.g. G = 1024, N = 4096: 5.9 us vs 28 us)

@@ -331,7 +331,7 @@ def test_auto_dispatch_regions():
     # r01_autotune_probe.jsonl); each shape must also scan exactly through AUTO
     want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 32768): "cluster", (4, 65536): "three_stage",
             (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
-            (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 23): "three_stage", (1, 1 << 24): "lookback",
+            (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 22): "three_stage", (1, 1 << 23): "lookback",
             (4096, 16384): "cascade_cta"}
     sb.autotune_clear()
     for (G, N), algo in want.items():

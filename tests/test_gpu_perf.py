@@ -121,3 +121,16 @@ def test_latency_bound_configs():
         xv, yv = x[:N], y[:N]
         us = _graph_us(lambda: sb.scan(xv, "add", out=yv))
         assert us <= FLOORS["g1_small_us_max"], (N, sb.plan(xv, yv), us)
+
+
+def test_mid_size_single_problem_rates():
+    # G = 1, N = 2^24 / 2^25 / 2^26: the L2-staged look-back's fill and drain are a large
+    # share of the call (round 2: 0.82 / 0.90 / 0.96 of copy with the lazy look-back)
+    x = torch.empty(1 << 26, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 6)
+    y = torch.empty_like(x)
+    for n, key in ((24, "g1_2e24_frac_min"), (25, "g1_2e25_frac_min"), (26, "g1_2e26_frac_min")):
+        N = 1 << n
+        xv, yv = x[:N], y[:N]
+        f = _frac(N, _graph_us(lambda: sb.scan(xv, "add", out=yv)) * 1e-3)
+        assert f >= FLOORS[key], (n, sb.plan(xv, yv), f)
