@@ -224,10 +224,12 @@ scan_status resolve_ws(void* ws, size_t ws_bytes, size_t need, cudaStream_t s, i
 // it, for A/B measurements)
 const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
 
-// look-back polling / tail options (A/B switches for on-box measurements)
-const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 4;
+// look-back options, A/B switches for on-box measurements (round 2):
+// SCANB200_LB_MODE=0 restores the round-1 speculative serialized look-back of the L2-staged
+// kernel, SCANB200_NO_KEEP_LAST=1 re-reads its last tiles, SCANB200_POLL_NS sets the first
+// back-off of a failed window poll
+const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 1;
 const bool g_keep_last = std::getenv("SCANB200_NO_KEEP_LAST") == nullptr;
-const int g_lb_tail = std::getenv("SCANB200_LB_TAIL") ? std::atoi(std::getenv("SCANB200_LB_TAIL")) : 1;
 const uint32_t g_poll_ns = (uint32_t)std::atoi(std::getenv("SCANB200_POLL_NS") ? std::getenv("SCANB200_POLL_NS") : "64");
 
 // debug timeline buffer for the look-back kernels (scan_debug_trace)
@@ -278,7 +280,6 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     p.lb_mode = g_lb_mode;
     p.keep_last = g_keep_last;
     p.poll_ns = g_poll_ns;
-    p.lb_tail = g_lb_tail;
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
 }
 

@@ -48,13 +48,11 @@ struct LookbackParams {
     bool pdl_first;     // cross-call programmatic launch (L2-staged kernel): CTAs may be
                         // scheduled while the stream's previous kernel drains and execute
                         // griddepcontrol.wait before their first global memory access
-    int lb_mode;        // 0: serial window polls; 1: window loads in flight together
-                        // (look_back_par); 2: as 1, and the L2-staged kernel uses the CTA's
-                        // own previous tile (look_back_rr)
+    int lb_mode;        // L2-staged kernel: 0 = round-1 speculative serialized look-back
+                        // (A/B only), otherwise the lazy round-robin look-back
     bool keep_last;     // L2-staged kernel: each CTA's last tile is scanned from the read-1
                         // ring slot (no second read on the kernel's critical tail)
-    uint32_t poll_ns;   // first back-off of a failed look-back poll (look_back_par)
-    int lb_tail;        // lb_mode 3: the CTA's last lb_tail tiles use look_back_rr
+    uint32_t poll_ns;   // first back-off of a failed look-back poll (look_back_par / _rr)
 };
 // u64 words per look-back descriptor slot.  A descriptor needs 1 (32-bit carries) or 2
 // (fp64 carries) words; one descriptor per 64-byte slot puts only two tiles on a 128-byte

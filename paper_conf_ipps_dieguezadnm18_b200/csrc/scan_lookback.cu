@@ -333,11 +333,6 @@ __device__ __forceinline__ typename Op::Carry look_back_rr(const LookbackParams&
     return run;
 }
 
-template <class Op, int M = LB_M>
-__device__ __forceinline__ typename Op::Carry look_back_any(const LookbackParams& p, int64_t t, uint32_t tag,
-                                                            uint32_t* stats = nullptr) {
-    return p.lb_mode == 1 ? look_back_par<Op, M>(p, t, tag, stats) : look_back<Op, M>(p, t, tag, stats);
-}
 
 // debug timeline (scan_debug_trace): stamp e of tile t with %globaltimer (ns)
 __device__ __forceinline__ void trace_stamp(const LookbackParams& p, int64_t t, int e) {
@@ -395,7 +390,7 @@ __device__ __forceinline__ void tile_body_smem(const LookbackParams& p, int64_t 
         const C aggc = Op::to_carry(agg);
         if (lane == 0) Desc<Op>::publish(p, tile, tag, has_head ? ST_P : ST_A, aggc);
         C carry = Op::cidentity();
-        if (!starts) carry = look_back_any<Op>(p, tile, tag);
+        if (!starts) carry = look_back<Op>(p, tile, tag);
         if (lane == 0) {
             if (!has_head) Desc<Op>::publish(p, tile, tag, ST_P, Op::capply(carry, aggc));
             *s_carry = carry;
@@ -420,11 +415,14 @@ __device__ __forceinline__ TileInfo classify(const LookbackParams& p, int64_t t,
 }
 
 // The last CTA to finish resets the counters and advances the epoch (wrap: clear all).
-// No fence before the count: the epoch only has to advance after every CTA READ it (at
-// its start, long before); a descriptor store of this launch still in flight carries this
-// launch's tag, which no later launch accepts, so the CTA need not wait for its stores
-// here (the next kernel is ordered after this grid's completion anyway).
-__device__ __forceinline__ void epilogue(const LookbackParams& p) {
+// No fence before the count in the common case: the epoch only has to advance after every
+// CTA READ it (at its start, long before); a descriptor store of this launch still in flight
+// carries this launch's tag, which no launch of the next ~2^30 accepts, so the CTA need not
+// wait for its stores here (the next kernel is ordered after this grid's completion anyway).
+// Only the launch that wraps the epoch (and clears every slot) fences first, so that none of
+// its own stores can land after the clear and survive into the next cycle of tags.
+__device__ __forceinline__ void epilogue(const LookbackParams& p, uint32_t tag) {
+    if (tag + 1u >= TAG_MASK) __threadfence();
     const uint32_t prev = atomicAdd(p.ctl + 1, 1u);
     if (prev == gridDim.x - 1) {
         __threadfence();
@@ -672,7 +670,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
             if (lane == 0) trace_stamp(p, t, 4);
-            if (!starts) carry = look_back_any<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+            if (!starts) carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
             mbar_wait(&s_p1[slot], ph);                   // this tile's aggregate is in the header
             SlotHdr<Op, WARPS>& h = s_hdr[slot];
             const bool has_head = h.has_head != 0u;
@@ -689,7 +687,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
+    if (threadIdx.x == 0) epilogue(p, tag);
 }
 
 // ---------------------------------------------------------------- two reads, L2-staged (variant 3)
@@ -751,9 +749,9 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         fence_mbar_init();
     }
     __syncthreads();
-    // the launch tag (an L2 round trip) is read only by the warps that publish or read
-    // descriptors, so the first read-1 bulk copies are not queued behind it
-    const uint32_t tag = ((warp >= NS && warp < NS + NR) || warp >= NS + NR + 2) ? read_tag(p) : 0u;
+    // the launch tag (an L2 round trip) is not read by the read-1 producer, so the first
+    // bulk copies are not queued behind it
+    const uint32_t tag = warp != NS + NR ? read_tag(p) : 0u;
     const T* in = (const T*)p.in;
 
     if (warp < NS) {
@@ -925,11 +923,11 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const int64_t t = (int64_t)blockIdx.x + i * (int64_t)gridDim.x;
             C carry = Op::cidentity();
             uint32_t stats[2] = {0u, 0u};
-            // mode 4 (lazy): the look-back starts once this tile's own aggregate is out --
+            // lazy (default, lb_mode != 0): the look-back starts once this tile's own aggregate is out --
             // its predecessors' aggregates arrive around the same time, so the window is
             // (nearly) complete at the first poll and no warp spins on descriptors that
             // cannot be ready yet (such polls slow the streaming reads they share L2 with)
-            const bool lazy = p.lb_mode == 4;
+            const bool lazy = p.lb_mode != 0;
             if (lazy) mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
             if (i < n_mine) {
                 if (lane == 0) trace_stamp(p, t, 4);
@@ -940,15 +938,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                     else
                         carry = look_back_par<Op, M>(p, t, tag, p.trace ? stats : nullptr);
                 } else if (((t * (int64_t)TILE) % p.N) != 0) {
-                    // mode 3: the serial (self-throttling) poll while the CTA streams, the
-                    // round-robin window with loads in flight for its last lb_tail tiles
-                    // (the kernel's drain, when no streaming traffic competes any more)
-                    const bool rr = p.lb_mode == 2 || (p.lb_mode == 3 && i + p.lb_tail >= n_mine);
-                    if (rr && i > 0 && (int64_t)gridDim.x - 1 <= 32 * M)
-                        carry = look_back_rr<Op, M>(p, t, i, gridDim.x, tag, s_incl, s_iseq, RING,
-                                                    p.trace ? stats : nullptr);
-                    else
-                        carry = look_back_any<Op, M>(p, t, tag, p.trace ? stats : nullptr);
+                    // mode 0 (round 1, kept for A/B): speculative serialized polls
+                    carry = look_back<Op, M>(p, t, tag, p.trace ? stats : nullptr);
                 }
             }
             if (!lazy) mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
@@ -974,7 +965,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
+    if (threadIdx.x == 0) epilogue(p, tag);
 }
 
 template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
@@ -1037,7 +1028,7 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
     if (s_seg) tile_body_smem<Op, true, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
     else       tile_body_smem<Op, false, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
+    if (threadIdx.x == 0) epilogue(p, tag);
 }
 
 // ---------------------------------------------------------------- one register tile per CTA
@@ -1085,7 +1076,7 @@ __device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t ti
         if (lane == 0) { trace_stamp(p, tile, 1); trace_stamp(p, tile, 4); }
         C carry = Op::cidentity();
         uint32_t stats[2] = {0u, 0u};
-        if (!starts) carry = look_back_any<Op>(p, tile, tag, p.trace ? stats : nullptr);
+        if (!starts) carry = look_back<Op>(p, tile, tag, p.trace ? stats : nullptr);
         if (lane == 0) {
             if (!has_head) Desc<Op>::publish(p, tile, tag, ST_P, Op::capply(carry, aggc));
             trace_stamp(p, tile, 2);
@@ -1113,7 +1104,7 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackPa
     if (ti.seg) regtile_body<Op, true, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
     else        regtile_body<Op, false, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p);
+    if (threadIdx.x == 0) epilogue(p, tag);
 }
 
 // ---------------------------------------------------------------- launchers

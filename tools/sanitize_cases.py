@@ -32,4 +32,16 @@ for dt, dist in (("i32", "i32"), ("f32", "f32s")):
         sb.shard_scan(x, torch.stack([t, t]), 1, 2, "add", "inclusive")
         torch.cuda.synchronize()
         print("ok", dt, N, G, flush=True)
+# the persistent L2-staged look-back over several rounds (lazy round-robin look-back with the
+# CTA-local previous prefix, kept tail tiles): more tiles than SMs, ragged last tile
+for dt, dist in (("i32", "i32"), ("f32", "f32s")):
+    N = 3 * 148 * 8192 + 1234
+    x = torch.empty(N, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, dist, 2)
+    if dt == "f32":
+        x = x.view(torch.float32)
+    for kind in ("inclusive", "exclusive"):
+        sb.scan(x, "add", kind, algo="lookback", param=3)
+        torch.cuda.synchronize()
+    print("ok multi-round", dt, N, flush=True)
 print("sanitize cases done")
