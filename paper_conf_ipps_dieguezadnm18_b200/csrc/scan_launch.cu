@@ -7,6 +7,7 @@
 // opt-in on each of them.  Both caches are keyed by device and guarded by one mutex.
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <utility>
@@ -86,9 +87,12 @@ cudaError_t launch_persistent(const void* func, void** args, int64_t tiles, int 
     // a cooperative launch guarantees that the whole grid is co-resident (or the launch
     // fails loudly, e.g. inside an SM-limited MPS / green context) instead of relying on
     // nothing else occupying the SMs
-    attr[n].id = cudaLaunchAttributeCooperative;
-    attr[n].val.cooperative = 1;
-    ++n;
+    static const bool coop = std::getenv("SCANB200_NO_COOP") == nullptr;   // A/B switch
+    if (coop) {
+        attr[n].id = cudaLaunchAttributeCooperative;
+        attr[n].val.cooperative = 1;
+        ++n;
+    }
     if (pdl) {
         attr[n].id = cudaLaunchAttributeProgrammaticStreamSerialization;
         attr[n].val.programmaticStreamSerializationAllowed = 1;

@@ -734,6 +734,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     __shared__ C s_incl[RING];
     __shared__ int64_t s_iseq[RING];
     const int warp = threadIdx.x >> 5, lane = lane_id();
+    if (threadIdx.x == 0) trace_stamp(p, blockIdx.x, 7);     // CTA entry (debug timeline)
     // every CTA is resident before a dependent grid can launch (launch_dependents counts
     // all of them), so the static round robin's inter-CTA waits cannot be starved of SMs;
     // the wait orders the previous kernel's writes (our input, the epoch) before any access
