@@ -53,3 +53,25 @@ def test_c3_shape_int32_full(kind):
     _check_streamed(xd, out, kind, np.int32, "int32 N=2^30 %s" % kind)
     del xd, out
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("G,N,op,dist,kind", [
+    (5, 3000017, "add", "i32", "inclusive"), (5, 3000017, "add", "i32", "exclusive"),
+    (5, 3000017, "add", "f32s", "inclusive"), (5, 3000017, "max", "i32", "exclusive"),
+    (3, 7 * 8192 * 148 + 5, "add", "u32", "inclusive"), (2048, 1 << 17, "add", "i32", "inclusive")])
+def test_lookback_multiround_segmented(G, N, op, dist, kind):
+    # the persistent L2-staged look-back over MANY rounds of the CTA round robin with problem
+    # starts inside tiles (segmented tiles publish P at once; the lazy look-back's window and
+    # the CTA-local previous prefix must both stop at problem boundaries); (2048, 2^17) is the
+    # paper-sweep point n = 17, checked in full
+    import inputs
+    from gpu_util import assert_parity
+    xd = device_inputs(dist, G * N, 0x5CA2018 + 11 + G).view(G, N)
+    assert sb.plan(xd, op=op, kind=kind) == ("lookback", 3)
+    out = sb.scan(xd, op, kind)
+    torch.cuda.synchronize()
+    dt = inputs.DIST_DTYPE[dist]
+    x = to_host(xd, dt).reshape(G, N)
+    assert_parity(to_host(out, dt).reshape(G, N), x, op, kind, label="multiround G=%d N=%d" % (G, N))
+    del xd, out
+    torch.cuda.empty_cache()
