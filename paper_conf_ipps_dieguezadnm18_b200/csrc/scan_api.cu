@@ -482,6 +482,50 @@ scan_status host_ctx(int dev, HostCtx** out) {
     return SCAN_OK;
 }
 
+// One staging unit: elements [off, off + n) of the flat batch = problems [g0, g0 + ng)
+// (whole problems, N <= piece) or piece j of problem g0 (long problems).
+struct HostUnit { int64_t off, n, g0, ng, j; };
+
+// Units of at most `piece` elements with a short RAMP at both ends of the call: the first
+// host->device copy and the last device->host copy cannot overlap anything (the pipeline
+// fills and drains), so they are made short -- piece/16, piece/4, then full pieces, then
+// piece/4, piece/16 (e2e).  Whole problems per unit when N <= piece; pieces
+// of one problem otherwise (a piece never spans two problems).
+std::vector<HostUnit> host_units(int64_t N, int64_t G, int64_t piece) {
+    std::vector<HostUnit> u;
+    const int64_t total = N * G;
+    const bool ramp = total > 2 * piece;
+    const int64_t r1 = std::max<int64_t>(piece / 16, 1), r2 = std::max<int64_t>(piece / 4, 1);
+    int64_t g = 0, e = 0, done = 0, j = 0;
+    while (done < total) {
+        const int64_t rem = total - done;
+        int64_t b = piece;
+        if (ramp) {
+            if (u.size() == 0) b = r1;
+            else if (u.size() == 1) b = r2;
+            else if (rem <= r1) b = rem;
+            else if (rem <= r1 + r2) b = rem - r1;
+            else if (rem <= piece + r1 + r2) b = rem - r1 - r2;
+        }
+        b = std::min(b, piece);
+        HostUnit h{};
+        if (N <= piece) {
+            const int64_t ng = std::min<int64_t>(std::max<int64_t>(b / N, 1), G - g);
+            h = HostUnit{g * N, ng * N, g, ng, 0};
+            g += ng;
+        } else {
+            const int64_t n = std::min<int64_t>(std::max<int64_t>(b, 1), N - e);
+            h = HostUnit{g * N + e, n, g, 1, j};
+            e += n;
+            ++j;
+            if (e == N) { e = 0; j = 0; ++g; }
+        }
+        done += h.n;
+        u.push_back(h);
+    }
+    return u;
+}
+
 scan_status host_pipeline(const void* in_host, void* out_host, int64_t N, int64_t G, scan_op op,
                           scan_dtype dt, scan_kind kind) {
     int dev = 0;
@@ -493,51 +537,39 @@ scan_status host_pipeline(const void* in_host, void* out_host, int64_t N, int64_
     const int64_t kPiece = host_piece();
     const int kSlots = host_slots();
     const bool pieces = N > kPiece;
-    const int64_t npieces = pieces ? (N + kPiece - 1) / kPiece : 0;
+    const std::vector<HostUnit> units = host_units(N, G, kPiece);
+    int64_t npieces = 0;
+    for (const HostUnit& h : units) npieces = std::max<int64_t>(npieces, h.j + 1);
     if (pieces && c->piece_cap < npieces) {
         if (c->piece_totals) cudaFree(c->piece_totals);
         c->piece_totals = nullptr;
         if (cudaMalloc(&c->piece_totals, npieces * 8) != cudaSuccess) { cudaGetLastError(); return SCAN_ERR_NO_MEMORY; }
         c->piece_cap = npieces;
     }
-    const int64_t per_group = pieces ? 1 : std::max<int64_t>(1, kPiece / N);
-    const int64_t units = pieces ? G * npieces : (G + per_group - 1) / per_group;
     const char* src = (const char*)in_host;
     char* dst = (char*)out_host;
-    for (int64_t u = 0; u < units; ++u) {
+    for (size_t u = 0; u < units.size(); ++u) {
         const int k = (int)(u % kSlots);
-        int64_t off, n_elem, j = 0, ng;
-        if (pieces) {
-            const int64_t g = u / npieces;
-            j = u % npieces;
-            off = g * N + j * kPiece;
-            n_elem = std::min<int64_t>(kPiece, N - j * kPiece);
-            ng = 1;
-        } else {
-            const int64_t g0 = u * per_group;
-            ng = std::min<int64_t>(per_group, G - g0);
-            off = g0 * N;
-            n_elem = ng * N;
-        }
-        if (u >= kSlots && cudaStreamWaitEvent(c->h2d, c->ev_out[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
-        if (cudaMemcpyAsync(c->slot[k], src + off * 4, n_elem * 4, cudaMemcpyHostToDevice, c->h2d) != cudaSuccess)
+        const HostUnit& h = units[u];
+        if (u >= (size_t)kSlots && cudaStreamWaitEvent(c->h2d, c->ev_out[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
+        if (cudaMemcpyAsync(c->slot[k], src + h.off * 4, h.n * 4, cudaMemcpyHostToDevice, c->h2d) != cudaSuccess)
             return SCAN_ERR_CUDA;
         if (cudaEventRecord(c->ev_in[k], c->h2d) != cudaSuccess) return SCAN_ERR_CUDA;
         if (cudaStreamWaitEvent(c->comp, c->ev_in[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
         if (pieces) {
             // piece j of a problem: three-stage scan whose carry folds the totals of pieces 0..j-1
             void* w = nullptr; size_t wb = 0;
-            st = cached_workspace(c->comp, FAM_CHUNKED, three_stage_bytes(n_elem, 1, 0), &w, &wb);
+            st = cached_workspace(c->comp, FAM_CHUNKED, three_stage_bytes(h.n, 1, 0), &w, &wb);
             if (st != SCAN_OK) return st;
-            st = run_three_stage(c->slot[k], c->slot[k], n_elem, 1, op, dt, kind, 0, w, c->piece_totals,
-                                 (int)j, c->comp, true, true, c->piece_totals + j);
+            st = run_three_stage(c->slot[k], c->slot[k], h.n, 1, op, dt, kind, 0, w, c->piece_totals,
+                                 (int)h.j, c->comp, true, true, c->piece_totals + h.j);
         } else {
-            st = run_algo(c->slot[k], c->slot[k], N, ng, op, dt, kind, SCAN_ALGO_AUTO, -1, nullptr, 0, c->comp);
+            st = run_algo(c->slot[k], c->slot[k], N, h.ng, op, dt, kind, SCAN_ALGO_AUTO, -1, nullptr, 0, c->comp);
         }
         if (st != SCAN_OK) return st;
         if (cudaEventRecord(c->ev_scan[k], c->comp) != cudaSuccess) return SCAN_ERR_CUDA;
         if (cudaStreamWaitEvent(c->d2h, c->ev_scan[k], 0) != cudaSuccess) return SCAN_ERR_CUDA;
-        if (cudaMemcpyAsync(dst + off * 4, c->slot[k], n_elem * 4, cudaMemcpyDeviceToHost, c->d2h) != cudaSuccess)
+        if (cudaMemcpyAsync(dst + h.off * 4, c->slot[k], h.n * 4, cudaMemcpyDeviceToHost, c->d2h) != cudaSuccess)
             return SCAN_ERR_CUDA;
         if (cudaEventRecord(c->ev_out[k], c->d2h) != cudaSuccess) return SCAN_ERR_CUDA;
     }
