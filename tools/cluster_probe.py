@@ -18,7 +18,7 @@ import paper_conf_ipps_dieguezadnm18_b200 as sb  # noqa: E402
 from g1_probe import graph_ms  # noqa: E402
 
 OTHERS = [("auto", -1), ("three_stage", 0), ("three_stage", 1), ("cascade_cta", -1), ("lookback", 10),
-          ("lookback", 11)]
+          ("lookback", 3)]
 CLUSTER = [32 * v + c for v in range(3) for c in (1, 2, 4, 8, 16)]
 
 
