@@ -34,3 +34,17 @@ def test_bench_world_size_mismatch_fails_loudly():
     r = _run(["--gpus", "2", "--dry-run"], env={"WORLD_SIZE": "1", "RANK": "0", "LOCAL_RANK": "0"})
     assert r.returncode == 2
     assert "WORLD_SIZE" in r.stderr
+
+
+def test_reference_arm_runs_on_cpu():
+    # the reference arm of this paper-only run is the CPU oracle (no GPU needed): one JSON
+    # line with impl=reference, the base contract's keys, cpu_baseline and a zero-copy e2e
+    r = _run(["--impl", "reference", "--steps", "2", "--warmup", "1"])
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["unit"] == "Gelem/s" and d["value"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["d2h_bytes_per_step"] == 0
+    assert d["higher_is_better"] is True and d["steps"] == 2 and d["warmup"] == 1
