@@ -24,7 +24,7 @@ for N in [1, 2, 3, 4, 8, 16, 32, 64, 100, 128, 255, 256, 257, 512, 600, 1000, 10
     xv, yv = x[:G * N].view(G, N), y[:G * N].view(G, N)
     res = []
     for algo, param in [("packed_warp", -1), ("packed_warp", 1024), ("packed_warp", 4096),
-                        ("lookback", 2), ("cascade_warp", -1)]:
+                        ("lookback", 2), ("lookback", 3), ("cascade_warp", -1)]:
         if algo == "cascade_warp" and N < 64:
             continue
         ms = t(xv, yv, algo, param)
