@@ -24,7 +24,7 @@
 //      on: the window of the grid - 1 predecessors is loaded in one round trip and the CTA's
 //      own previous tile supplies the inclusive prefix from shared memory) while the data
 //      waits in L2; read 2 (L2 -> smem) feeds 8 scanner warps that add the carry and store
-//      (the CTA's last tile is scanned from its read-1 slot).  The next round's read 1 is
+//      (the CTA's last two tiles are scanned from their read-1 slots).  The next round's read 1 is
 //      L2-prefetched (UBLKPF).  ~100 % of measured copy from 2^27 on, 0.82 / 0.90 at 2^24 / 2^25.
 //   0/1 lookback_pipelined_kernel -- persistent, one read: a producer warp streams 64 / 32
 //      KiB tiles into a 3-slot TMA ring, 16 / 8 consumer warps scan each staged tile in two
