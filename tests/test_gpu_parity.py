@@ -167,25 +167,26 @@ def test_determinism_ints_and_three_stage_f32():
     assert all(np.array_equal(outs[0], o) for o in outs[1:])
 
 
-def test_cuda_graph_replay_self_cleaning():
+@pytest.mark.parametrize("param,N,G", [(-1, 300001, 2), (3, (1 << 23) + 123, 1), (3, 3000017, 3)])
+def test_cuda_graph_replay_self_cleaning(param, N, G):
     # the look-back descriptors are reset-free (epoch tags): replaying a captured launch
-    # must stay correct without any memset between replays
-    N, G = 300001, 2
+    # must stay correct without any memset between replays -- also for the cooperative,
+    # persistent L2-staged kernel over many rounds (param 3)
     x = inputs.generate("f32s", N * G, 3).reshape(G, N)
     xd = to_device(x)
     out = torch.empty_like(xd)
     s = torch.cuda.Stream()
     with torch.cuda.stream(s):
-        sb.scan(xd, "add", out=out, algo="lookback")       # warm-up (workspace allocation)
+        sb.scan(xd, "add", out=out, algo="lookback", param=param)       # warm-up (workspace allocation)
     torch.cuda.synchronize()
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g, stream=s):
-        sb.scan(xd, "add", out=out, algo="lookback")
+        sb.scan(xd, "add", out=out, algo="lookback", param=param)
     for _ in range(20):
         out.zero_()
         g.replay()
     torch.cuda.synchronize()
-    assert_parity(to_host(out, np.float32), x, "add", "inclusive", label="graph")
+    assert_parity(to_host(out, np.float32), x, "add", "inclusive", label="graph param=%d" % param)
 
 
 def test_epoch_wrap_with_caller_workspace():
