@@ -81,7 +81,7 @@ def main():
     outdir = os.path.join(ROOT, "gpurun_out")
     os.makedirs(outdir, exist_ok=True)
     res = {"src_sha256": bench.source_sha256(),
-           "captured": datetime.datetime.utcnow().strftime("%Y-%m-%dT%H:%MZ"),
+           "captured": datetime.datetime.now(datetime.timezone.utc).strftime("%Y-%m-%dT%H:%MZ"),
            "how": "ncu --set full --clock-control none, one launch after 2 warm-up launches, cold caches",
            "cases": {}}
     for name in CASES:
