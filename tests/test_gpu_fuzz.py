@@ -39,3 +39,28 @@ def test_random_cases(seed):
         assert_parity(to_host(out, NP[dt]).reshape(G, N), x[off:].reshape(G, N), op, kind,
                       label="fuzz seed=%d case=%d %s/%d %s %s %s N=%d G=%d off=%d" % (
                           seed, case, algo, param, op, dt, kind, N, G, off))
+
+
+@pytest.mark.parametrize("seed", range(int(__import__("os").environ.get("SCANB200_FUZZ_LARGE_SEEDS", "3"))))
+def test_random_multiround_lookback(seed):
+    # the persistent L2-staged look-back over many rounds of its round robin (lazy look-back,
+    # CTA-local previous prefix, kept tail tiles): random G x N up to 4*10^7 elements, random
+    # ops / dtypes / kinds / pointer offsets (offsets take the unaligned, non-TMA path)
+    rng = random.Random(7000 + seed)
+    for case in range(8):
+        total = rng.randint(2_000_000, 40_000_000)
+        G = rng.choice([1, 1, 2, 3, rng.randint(4, 64), rng.randint(64, 2000)])
+        N = max(1, total // G)
+        op, dt = rng.choice(COMBOS)
+        kind = rng.choice(["inclusive", "exclusive"])
+        param = rng.choice([3, 3, -1])
+        off = rng.choice([0, 0, 0, 1, 3])
+        x = inputs.generate(DIST[dt], N * G + off, seed=seed * 100 + case)
+        base = to_device(x)
+        xin = base[off: off + N * G].view(G, N)
+        out = torch.empty(N * G + 4, dtype=base.dtype, device="cuda")[off: off + N * G].view(G, N)
+        sb.scan(xin, op, kind, out=out, algo="lookback", param=param)
+        torch.cuda.synchronize()
+        assert_parity(to_host(out, NP[dt]).reshape(G, N), x[off:].reshape(G, N), op, kind,
+                      label="fuzz-large seed=%d case=%d lookback/%d %s %s %s N=%d G=%d off=%d" % (
+                          seed, case, param, op, dt, kind, N, G, off))
