@@ -148,7 +148,8 @@ KERNEL_NAMES = {"lookback": "lookback_*_kernel (decoupled look-back)",
                 "cascade_warp": "warp_cascade_kernel (one warp per problem, cascade)",
                 "three_stage": "chunk_reduce + aux_scan + chunk_scan kernels",
                 "packed_warp": "packed_warp_kernel (k short problems per warp, segmented)",
-                "cluster": "cluster_scan_kernel (one thread-block cluster per problem, DSMEM aggregates)"}
+                "cluster": "cluster_scan_kernel (one thread-block cluster per problem, DSMEM aggregates)",
+                "fused": "fused_grid_kernel (three stages in one cooperative launch, tiles in registers)"}
 
 
 def plan(x: torch.Tensor, out: torch.Tensor | None = None, op: str = "add",

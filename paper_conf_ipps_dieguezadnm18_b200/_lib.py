@@ -15,7 +15,8 @@ LIB_PATH = os.path.join(_HERE, "libscanb200.so")
 # enum values of include/scan_b200.h
 OPS = {"add": 0, "max": 1}
 KINDS = {"inclusive": 0, "exclusive": 1}
-ALGOS = {"auto": 0, "lookback": 1, "cascade_cta": 2, "cascade_warp": 3, "three_stage": 4, "packed_warp": 5, "cluster": 6}
+ALGOS = {"auto": 0, "lookback": 1, "cascade_cta": 2, "cascade_warp": 3, "three_stage": 4, "packed_warp": 5, "cluster": 6,
+         "fused": 7}
 STATUS = {0: "SCAN_OK", 1: "SCAN_ERR_INVALID_ARG", 2: "SCAN_ERR_UNSUPPORTED", 3: "SCAN_ERR_CUDA",
           4: "SCAN_ERR_NCCL", 5: "SCAN_ERR_NO_MEMORY", 6: "SCAN_ERR_NO_DEVICE"}
 

@@ -76,6 +76,13 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // (2^15 < N <= 2^16 at G = 1: the two-launch chain 3.6 us vs the cluster 3.9-4.0 us once
     //  both use programmatic launch, profiles/r01_g1_probe_cluster_boundary.jsonl)
     if (G <= 64 && N <= 32768) return SCAN_ALGO_CLUSTER;
+    // one problem of 2.5 M .. ~4.8 M elements (as many 8192-element tiles as CTAs fit at once):
+    // the three stages fused into one cooperative launch with every tile held in registers
+    // across one grid barrier -- one read instead of two, one launch instead of two or three
+    // (4.7 M: 8.6 vs 13.3 us three-stage, 11.7 us look-back; 2^22: 8.4 vs 9.5 us;
+    // profiles/r02_fused_probe.jsonl); below 2.5 M the two-launch chain is faster
+    if (G == 1 && N > (int64_t(5) << 19) && N <= fused_max_tiles(OpCode::AddF32) * fused_tile_elems())
+        return SCAN_ALGO_FUSED;
     // three-stage up to ~7 x 2^20 elements: the second read of the input still hits L2, and
     // the chain beats the L2-staged look-back's fill/drain there (6 x 2^20: 12.9 vs 13.5 us);
     // the lazy look-back wins from 2^23 (15.0 vs 15.6 us i32, 14.9 vs 15.4 us f32;
@@ -173,6 +180,10 @@ size_t lookback_bytes(int64_t total, int variant, bool split) {
     int64_t tile = lookback_tile_elems(variant);
     int64_t tiles = (total + tile - 1) / tile;
     return kCtlBytes + kLbSlotBytes * (size_t)tiles;
+}
+size_t fused_bytes(int64_t N, int64_t G) {
+    const int64_t tile = fused_tile_elems();
+    return kCtlBytes + align_up((size_t)((N * G + tile - 1) / tile) * 8, 256);
 }
 size_t three_stage_bytes(int64_t N, int64_t G, int64_t K) {
     int64_t chunk = three_stage_chunk(N, G, K);
@@ -368,8 +379,9 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         if (ws || !tuned_choice(tune_key(N, G, aligned, op, dt, kind), &algo, &param)) {
             algo = choose_algo(N, G, aligned);
             // a caller workspace is sized and laid out for the look-back family
-            // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage scratch into it
-            if (ws && algo == SCAN_ALGO_THREE_STAGE) algo = SCAN_ALGO_LOOKBACK;
+            // (scan_workspace_bytes(AUTO)); never let AUTO put three-stage or fused scratch
+            // (untagged values the look-back could misread) into it
+            if (ws && (algo == SCAN_ALGO_THREE_STAGE || algo == SCAN_ALGO_FUSED)) algo = SCAN_ALGO_LOOKBACK;
             param = -1;
         }
     }
@@ -414,6 +426,24 @@ scan_status run_algo(const void* in, void* out, int64_t N, int64_t G, scan_op op
         ChunkParams p = chunk_params(in, out, N, G, kind);
         p.pdl_first = g_cross_pdl;
         return from_cuda(launch_cluster_scan(opcode(op, dt), p, variant, csize, s));
+    }
+    case SCAN_ALGO_FUSED: {
+        const int64_t tile = fused_tile_elems();
+        const int64_t tiles = (N * G + tile - 1) / tile;
+        if (!(G == 1 || N % tile == 0)) return SCAN_ERR_UNSUPPORTED;
+        if (tiles > fused_max_tiles(opcode(op, dt))) return SCAN_ERR_UNSUPPORTED;
+        void* w = nullptr;
+        size_t wb = 0;
+        scan_status st = resolve_ws(ws, ws_bytes, fused_bytes(N, G), s, FAM_CHUNKED, &w, &wb);
+        if (st != SCAN_OK) return st;
+        FusedParams p{};
+        p.in = in; p.out = out; p.total = N * G;
+        p.tiles_per_problem = G == 1 ? tiles : N / tile;
+        p.aux = (uint64_t*)((char*)w + kCtlBytes);
+        p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0);
+        p.exclusive = kind == SCAN_EXCLUSIVE;
+        p.pdl_first = g_cross_pdl;
+        return from_cuda(launch_fused(opcode(op, dt), p, s));
     }
     case SCAN_ALGO_THREE_STAGE: {
         void* w = nullptr;
@@ -637,6 +667,7 @@ size_t scan_workspace_bytes(int64_t N, int64_t G, scan_op op, scan_dtype dtype, 
         return lookback_bytes(N * G, variant, split_desc(op, dtype));
     }
     if (algo == SCAN_ALGO_THREE_STAGE) return three_stage_bytes(N, G, param);
+    if (algo == SCAN_ALGO_FUSED) return fused_bytes(N, G);
     return kCtlBytes;
 }
 
@@ -645,7 +676,7 @@ scan_status scan_batch_ex(const void* in, void* out, int64_t N, int64_t G, scan_
                           size_t workspace_bytes, void* stream) {
     NvtxRange nvtx_range("scan_batch");
     if (!valid_enums(op, dtype, kind)) return SCAN_ERR_INVALID_ARG;
-    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_CLUSTER) return SCAN_ERR_UNSUPPORTED;
+    if (algo < SCAN_ALGO_AUTO || algo > SCAN_ALGO_FUSED) return SCAN_ERR_UNSUPPORTED;
     int64_t total = 0;
     scan_status st = check_shape(N, G, &total);
     if (st != SCAN_OK) return st;
@@ -683,6 +714,7 @@ scan_status scan_autotune(const void* in, void* out, int64_t N, int64_t G, scan_
     if (G >= 64 || N <= (int64_t(1) << 16)) cand.push_back({SCAN_ALGO_CASCADE_CTA, -1});
     if (G >= 256 && N <= (int64_t(1) << 16)) cand.push_back({SCAN_ALGO_CASCADE_WARP, -1});
     if (aligned && N < 1024) cand.push_back({SCAN_ALGO_PACKED_WARP, -1});
+    cand.push_back({SCAN_ALGO_FUSED, -1});                   // rejects ineligible shapes itself
     if (N <= (int64_t(1) << 20) && G * kMaxClusterCtas <= 0x7FFFFFFFll)
         for (int v = 0; v < 3; ++v)
             for (int c : {2, 4, 8, 16}) cand.push_back({SCAN_ALGO_CLUSTER, 32 * v + c});

@@ -137,6 +137,23 @@ cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s);
 constexpr int kMaxClusterCtas = 16;
 int64_t cluster_tile_elems(int variant);
 cudaError_t launch_cluster_scan(OpCode op, const ChunkParams& p, int variant, int csize, cudaStream_t s);
+// ---------------------------------------------------------------- fused three stages
+// scan_fused.cu: Stage 1 -> grid barrier -> Stage 2 fold -> Stage 3 in ONE cooperative
+// launch, one 8192-element tile per CTA held in registers (latency-bound totals).
+struct FusedParams {
+    const void* in;
+    void* out;
+    int64_t total;              // G * N
+    int64_t tiles_per_problem;  // N / tile when N is a multiple of the tile, else (G == 1) all tiles
+    uint64_t* aux;              // [tiles] 8-byte aggregate slots
+    bool vec;
+    bool exclusive;
+    bool pdl_first;
+};
+int64_t fused_tile_elems();
+int64_t fused_max_tiles(OpCode op);  // co-resident CTAs on the current device (0 on error)
+cudaError_t launch_fused(OpCode op, const FusedParams& p, cudaStream_t s);
+
 // Fused exchange with an empty local portion (no Stage 3 CTAs): one CTA waits for the
 // flags of ranks < rank and acknowledges them, so peers never wait on this rank.
 cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s);

@@ -332,7 +332,7 @@ def test_auto_dispatch_regions():
     # r01_autotune_probe.jsonl); each shape must also scan exactly through AUTO
     want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 32768): "cluster", (4, 65536): "three_stage",
             (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
-            (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 22): "three_stage", (1, 1 << 23): "lookback",
+            (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 21): "three_stage", (1, 1 << 22): "fused", (1, 1 << 23): "lookback",
             (4096, 16384): "cascade_cta"}
     sb.autotune_clear()
     for (G, N), algo in want.items():
@@ -389,7 +389,8 @@ def test_autotune_with_caller_workspace():
 @pytest.mark.parametrize("algo,G,N", [("cascade_cta", 512, 8192), ("cascade_warp", 2000, 1000),
                                       ("packed_warp", 20000, 100), ("cluster", 3, 30000),
                                       ("three_stage", 1, 1 << 20), ("auto", 4096, 4096),
-                                      ("lookback/3", 1, 1 << 22), ("lookback/3", 3, 1000003)])
+                                      ("lookback/3", 1, 1 << 22), ("lookback/3", 3, 1000003),
+                                      ("fused", 1, 1 << 22), ("fused", 4, 1 << 16)])
 def test_back_to_back_ordering(algo, G, N):
     # the single-kernel families and Stage 1 are launched as programmatic dependents of the
     # stream's previous kernel and wait before their first access: chains of dependent
@@ -410,3 +411,32 @@ def test_back_to_back_ordering(algo, G, N):
     torch.cuda.synchronize()
     got = to_host(xd, np.int32)
     assert np.array_equal(got, ref), algo
+
+
+@pytest.mark.parametrize("op,dt", COMBOS)
+def test_fused_family(op, dt):
+    # SCAN_ALGO_FUSED: the three stages in one cooperative launch, one 8192-element tile per
+    # CTA held in registers across one grid barrier.  One problem of any N (ragged last
+    # tile), or G problems with N a multiple of the tile; unaligned pointers take the
+    # scalar path; shapes beyond the co-resident capacity or with ragged multi-problem
+    # layouts are rejected (SCAN_ERR_UNSUPPORTED), never mis-scanned.
+    shapes = [(1, 1), (1, 8191), (1, 8193), (1, 1000003), (1, 4 * 1024 * 1024 + 5), (3, 8192), (5, 8192 * 9),
+              (64, 65536)]
+    for G, N in shapes:
+        x = inputs.generate(DIST[dt], G * N, seed=G * 31 + N % 977).reshape(G, N)
+        for kind in ("inclusive", "exclusive"):
+            got = _run(x, op, kind, "fused")
+            assert_parity(got, x, op, kind, label="fused %s %s %s G=%d N=%d" % (op, dt, kind, G, N))
+    # unaligned base pointers
+    x = inputs.generate(DIST[dt], 300001 + 1, seed=5)
+    base = to_device(x)
+    xin = base[1:]
+    out = torch.empty(300001 + 4, dtype=base.dtype, device="cuda")[3:300004]
+    sb.scan(xin, op, "inclusive", out=out, algo="fused")
+    torch.cuda.synchronize()
+    assert_parity(to_host(out, NP[dt]), x[1:], op, "inclusive", label="fused unaligned")
+    # ineligible: ragged N with G > 1, and more tiles than CTAs fit at once
+    with pytest.raises(sb.ScanError):
+        sb.scan(torch.zeros((3, 10000), dtype=TORCH[dt], device="cuda"), op, algo="fused")
+    with pytest.raises(sb.ScanError):
+        sb.scan(torch.zeros(1 << 26, dtype=TORCH[dt], device="cuda"), op, algo="fused")
