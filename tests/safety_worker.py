@@ -3,7 +3,8 @@ script in a fresh process, so every kernel's first-use setup -- the per-device s
 memory opt-in and occupancy cache of scan_launch.cu -- happens under contention).
 
 T host threads, each with its own CUDA stream, issue look-back (persistent cooperative
-grids that each want every SM), cluster, three-stage and cascade scans at the same time.
+grids that each want every SM), fused (a cooperative grid with a grid barrier), cluster,
+three-stage and cascade scans at the same time.
 Two persistent grids on two streams must never deadlock by splitting the SMs between
 them; every result must be exact.  Prints "ok" or the first failure.
 """
@@ -20,7 +21,7 @@ from gpu_util import to_host
 
 CASES = [("lookback", 3, 1, 1 << 24), ("lookback", 0, 1, 1 << 23), ("lookback", 1, 3, 1000003),
          ("lookback", 2, 5000, 100), ("cluster", -1, 3, 30000), ("three_stage", 0, 2, 1 << 20),
-         ("cascade_cta", -1, 512, 8192), ("lookback", 3, 2, 1 << 23)]
+         ("cascade_cta", -1, 512, 8192), ("lookback", 3, 2, 1 << 23), ("fused", -1, 1, 3 << 20)]
 
 
 def worker(k, errors, iters):

@@ -109,7 +109,7 @@ def test_concurrent_first_use_and_streams():
     # opt-in / occupancy caches under contention), and persistent cooperative grids on 8
     # streams at once; a deadlock would hang, so the worker runs under a time limit
     env = dict(os.environ, PYTHONPATH=os.pathsep.join([os.path.dirname(HERE), HERE]))
-    r = subprocess.run([sys.executable, os.path.join(HERE, "safety_worker.py"), "8", "6"], env=env,
+    r = subprocess.run([sys.executable, os.path.join(HERE, "safety_worker.py"), "9", "6"], env=env,
                        capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stderr[-3000:]
     assert r.stdout.strip().splitlines()[-1] == "ok", r.stdout[-2000:]
