@@ -102,3 +102,15 @@ def test_lookback_variants_match_library():
     assert _lib.LOOKBACK_VARIANTS == valid
     par = open(os.path.join(os.path.dirname(__file__), "test_gpu_parity.py")).read()
     assert '@pytest.mark.parametrize("variant", _lib.LOOKBACK_VARIANTS)\ndef test_lookback_variants' in par
+
+
+def test_binding_enums_match_header():
+    # the ctypes binding's enum tables are the header's values (ops, kinds, algos, statuses)
+    from paper_conf_ipps_dieguezadnm18_b200 import _lib
+    src = open(os.path.join(ROOT, "include", "scan_b200.h")).read()
+    vals = {m.group(1): int(m.group(2)) for m in re.finditer(r"\b(SCAN_[A-Z0-9_]+)\s*=\s*(\d+)", src)}
+    assert {k: vals["SCAN_ALGO_" + k.upper()] for k in _lib.ALGOS} == _lib.ALGOS
+    assert {k: vals["SCAN_OP_" + k.upper()] for k in _lib.OPS} == _lib.OPS
+    assert {k: vals["SCAN_" + k.upper()] for k in _lib.KINDS} == _lib.KINDS
+    assert {vals[name]: name for name in _lib.STATUS.values()} == _lib.STATUS
+    assert len([k for k in vals if k.startswith("SCAN_ALGO_")]) == len(_lib.ALGOS)
