@@ -5,7 +5,8 @@ copy, and the same for torch.cumsum.
 
     python tools/paper_sweep.py batch [n0]   # 2^28 int32 as G = 2^28/N problems of N = 2^n,
                                              # n = n0..28 (PAPER.md:241, 249, 261 [Figs. 9-12])
-    python tools/paper_sweep.py g1 [n0]      # G = 1, N = 2^n, n = n0..30 (PAPER.md:255, 259 [Fig. 11])
+    python tools/paper_sweep.py g1 [n0 [n1]] # G = 1, N = 2^n, n = n0..n1 (default 30; up to 33 on one B200)
+                                             # (PAPER.md:255, 259 [Fig. 11])
 
 Device time per call: 20 calls captured in a CUDA graph and replayed between two events
 (so the small, latency-bound points are not host-launch bound)."""
@@ -48,7 +49,7 @@ def device_ms(fn, reps=20):
 def main():
     mode = sys.argv[1] if len(sys.argv) > 1 else "batch"
     n0 = int(sys.argv[2]) if len(sys.argv) > 2 else 10
-    n1 = 28 if mode == "batch" else 30
+    n1 = 28 if mode == "batch" else (int(sys.argv[3]) if len(sys.argv) > 3 else 30)
     total_max = 1 << n1
     x = torch.empty(total_max, dtype=torch.int32, device="cuda")
     inputs.fill_device(x, "i32", 2018)
