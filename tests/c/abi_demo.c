@@ -1,5 +1,6 @@
 /* abi_demo.c -- the C-ABI used from plain C (no Python, no torch): allocate with the CUDA
- * runtime, fill a batch, call scan_batch / scan_batch_ex / scan_batch_host /
+ * runtime, fill a batch, call scan_batch / scan_batch_ex (every kernel family) /
+ * scan_plan_ex / scan_batch_host /
  * scan_shard_totals + scan_shard_scan, and check the results against a sequential loop
  * written here (integer add: exact).  Built and run by tests/test_gpu_c_abi.py. */
 #include <stdint.h>
@@ -47,6 +48,22 @@ int main(void) {
         cudaMemcpy(hy, dy, n * 4, cudaMemcpyDeviceToHost);
         if (verify(hx, hy, N, G, 1, "scan_batch_ex")) return 1;
     }
+
+    /* the remaining families through scan_batch_ex, and what scan_plan_ex reports for AUTO */
+    for (int algo = SCAN_ALGO_PACKED_WARP; algo <= SCAN_ALGO_CLUSTER; ++algo) {
+        CHECK(scan_batch_ex(dx, dy, N, G, SCAN_OP_ADD, SCAN_I32, SCAN_INCLUSIVE, (scan_algo)algo, -1, NULL, 0, NULL));
+        cudaMemcpy(hy, dy, n * 4, cudaMemcpyDeviceToHost);
+        if (verify(hx, hy, N, G, 0, "scan_batch_ex")) return 1;
+    }
+    CHECK(scan_batch_ex(dx, dy, N, 1, SCAN_OP_ADD, SCAN_I32, SCAN_EXCLUSIVE, SCAN_ALGO_FUSED, -1, NULL, 0, NULL));
+    cudaMemcpy(hy, dy, N * 4, cudaMemcpyDeviceToHost);
+    if (verify(hx, hy, N, 1, 1, "fused")) return 1;
+    if (scan_batch_ex(dx, dy, N, G, SCAN_OP_ADD, SCAN_I32, SCAN_INCLUSIVE, SCAN_ALGO_FUSED, -1, NULL, 0, NULL)
+        != SCAN_ERR_UNSUPPORTED) return 3;                  /* ragged N with G > 1 */
+    int algo_auto = -1;
+    int64_t param_auto = 0;
+    CHECK(scan_plan_ex(N, G, SCAN_OP_ADD, SCAN_I32, SCAN_INCLUSIVE, dx, dy, &algo_auto, &param_auto));
+    if (algo_auto <= SCAN_ALGO_AUTO || algo_auto > SCAN_ALGO_FUSED) return 3;
 
     CHECK(scan_batch_host(hx, hy, N, G, SCAN_OP_ADD, SCAN_I32, SCAN_INCLUSIVE));
     if (verify(hx, hy, N, G, 0, "scan_batch_host")) return 1;
