@@ -83,11 +83,11 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // profiles/r02_fused_probe.jsonl); below 2.5 M the two-launch chain is faster
     if (G == 1 && N > (int64_t(5) << 19) && N <= fused_max_tiles(OpCode::AddF32) * fused_tile_elems())
         return SCAN_ALGO_FUSED;
-    // three-stage up to ~7 x 2^20 elements: the second read of the input still hits L2, and
-    // the chain beats the L2-staged look-back's fill/drain there (6 x 2^20: 12.9 vs 13.5 us);
-    // the lazy look-back wins from 2^23 (15.0 vs 15.6 us i32, 14.9 vs 15.4 us f32;
-    // profiles/r02_g1_boundary.jsonl)
-    if (G <= 64 && N * G <= (int64_t(7) << 20) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
+    // three-stage up to 2^22 elements (two launches: the second read of the input still
+    // hits L2); above, the three-launch form loses to the lazy look-back (5 x 2^20: 12.3 /
+    // 13.2 us against 12.5 / 12.5 us i32 / f32; 7 x 2^20: 15.5 against 14.2 / 15.0 us;
+    // profiles/r02_fused_probe_tpc2_REVERTED.jsonl)
+    if (G <= 64 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
     // a few hundred to a few thousand problems of moderate length (scan_autotune over a
     // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA
     // beat the flat look-back 1.1-4.8x there (e.g. G = 1024, N = 4096: 5.9 us vs 28 us)
