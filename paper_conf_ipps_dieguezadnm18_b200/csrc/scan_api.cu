@@ -67,6 +67,16 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // (N = 4096 exactly: one warp per problem 102 % vs one CTA 93 % of copy at G = 2^16,
     //  tools/n12_probe.py)
     if (rows_aligned && G >= 4096 && N > 4096) return SCAN_ALGO_CASCADE_CTA;
+    // hundreds to thousands of problems just above 2^16 elements, and a few thousand up to
+    // ~2^18: one CTA per problem beats the flat look-back there, by 3-74 % where problem
+    // starts fall inside look-back tiles (N not a multiple of 8192: every problem's first
+    // tile needs its own look-back, the CTAs fall out of step and the round-robin
+    // look-backs re-poll), ~equal on tile-aligned N (tools/cascade_boundary_probe.py,
+    // profiles/r02_cascade_boundary.jsonl); from 2^18 on at G < 2400 the look-back wins
+    if (rows_aligned && N > 65536 &&
+        ((G >= 300 && N <= 100000) || (G >= 1024 && N <= 131072) ||
+         (G >= 2048 && (G >= 2400 || N < 262144))))
+        return SCAN_ALGO_CASCADE_CTA;
     if (rows_aligned && G >= 1184 && N >= 768 && N <= 4096) return SCAN_ALGO_CASCADE_WARP;
     // few short / medium problems (latency bound, tools/cluster_probe.py on B200,
     // profiles/r01_cluster_probe.jsonl): one CTA per problem up to 8192 elements

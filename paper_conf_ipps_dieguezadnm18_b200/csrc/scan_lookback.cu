@@ -718,6 +718,26 @@ __device__ __forceinline__ typename Op::T warp_reduce_rows(const typename Op::T*
     return acc;
 }
 
+// The same over the chunk's elements at tile offsets >= first only (o0 = the chunk's tile
+// offset); the earlier ones belong to the previous problem.  Commutative ops only (add, max).
+template <class Op, int V>
+__device__ __forceinline__ typename Op::T warp_reduce_rows_from(const typename Op::T* srow, int o0, int first) {
+    using T = typename Op::T;
+    const int lane = lane_id();
+    T acc = Op::identity();
+#pragma unroll
+    for (int j = 0; j < V; ++j) {
+        Row4<T> x = row_from_u4<T>(lds_v4(srow + j * 128 + lane * 4));
+        const int o = o0 + j * 128 + lane * 4;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (o + q >= first) acc = Op::apply(acc, x.v[q]);
+    }
+#pragma unroll
+    for (int d = 16; d >= 1; d >>= 1) acc = Op::apply(acc, from_bits<T>(__shfl_xor_sync(FULL, to_bits<T>(acc), d)));
+    return acc;
+}
+
 template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
 __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kernel(LookbackParams p, int64_t num_tiles) {
     using T = typename Op::T;
@@ -808,11 +828,19 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             for (int k = rr; k < NS; k += NR) {
                 const T* srow = bufR + (size_t)sR * TILE + k * WCH;
                 T tot; bool fl = false;
-                if (seg) {
-                    const bool small = p.N < TILE;
-                    const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
+                if (seg && p.N >= TILE) {
+                    // N >= TILE: the tile holds exactly one problem start, at `first`; the
+                    // chunk that contains it folds only the elements from there on (the new
+                    // problem's head), every other chunk is a plain total -- a masked
+                    // reduction instead of a full segmented scan (which left seg tiles' A
+                    // ~1.7 us late and every look-back behind them re-polling)
+                    const int first = (int)(p.N - r);
+                    const int lo = k * WCH;
+                    fl = first >= lo && first < lo + WCH;
+                    tot = fl ? warp_reduce_rows_from<Op, V>(srow, lo, first) : warp_reduce_rows<Op, V>(srow);
+                } else if (seg) {
                     WarpTileP<Op, V> st;
-                    st.template pass1<true>(srow, k * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+                    st.template pass1<true>(srow, k * WCH, true, (uint32_t)r, (uint32_t)p.N, -1);
                     tot = st.wtot; fl = st.wfl;
                 } else {
                     tot = warp_reduce_rows<Op, V>(srow);

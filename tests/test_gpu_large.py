@@ -58,7 +58,8 @@ def test_c3_shape_int32_full(kind):
 @pytest.mark.parametrize("G,N,op,dist,kind", [
     (5, 3000017, "add", "i32", "inclusive"), (5, 3000017, "add", "i32", "exclusive"),
     (5, 3000017, "add", "f32s", "inclusive"), (5, 3000017, "max", "i32", "exclusive"),
-    (3, 7 * 8192 * 148 + 5, "add", "u32", "inclusive"), (2048, 1 << 17, "add", "i32", "inclusive")])
+    (3, 7 * 8192 * 148 + 5, "add", "u32", "inclusive"), (2048, 1 << 17, "add", "i32", "inclusive"),
+    (2048, 65540, "add", "i32", "exclusive"), (700, 200003, "add", "f32s", "inclusive")])
 def test_lookback_multiround_segmented(G, N, op, dist, kind):
     # the persistent L2-staged look-back over MANY rounds of the CTA round robin with problem
     # starts inside tiles (segmented tiles publish P at once; the lazy look-back's window and
@@ -67,8 +68,8 @@ def test_lookback_multiround_segmented(G, N, op, dist, kind):
     import inputs
     from gpu_util import assert_parity
     xd = device_inputs(dist, G * N, 0x5CA2018 + 11 + G).view(G, N)
-    assert sb.plan(xd, op=op, kind=kind) == ("lookback", 3)
-    out = sb.scan(xd, op, kind)
+    # forced: AUTO sends (2048, 2^17) to one CTA per problem since round 2 session 3
+    out = sb.scan(xd, op, kind, algo="lookback", param=3)
     torch.cuda.synchronize()
     dt = inputs.DIST_DTYPE[dist]
     x = to_host(xd, dt).reshape(G, N)

@@ -16,7 +16,8 @@ import paper_conf_ipps_dieguezadnm18_b200 as sb  # noqa: E402
 from gpu_util import COMBOS, DIST, NP, assert_parity, to_device, to_host  # noqa: E402
 
 SHAPES = [(1, 3000), (3, 5000), (100, 333), (8193, 5), (65536 + 17, 3), (1 << 20, 1),
-          ((1 << 23) + 123, 1), (3000017, 3), (1 << 17, 2048), (1 << 24, 1), (7777777, 2)]
+          ((1 << 23) + 123, 1), (3000017, 3), (1 << 17, 2048), (1 << 24, 1), (7777777, 2),
+          (65540, 2048), (200003, 700), (8191 * 3, 1001)]
 
 for v in [int(a) for a in sys.argv[1:]]:
     n = 0
