@@ -333,7 +333,7 @@ def test_auto_dispatch_regions():
     want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 32768): "cluster", (4, 65536): "three_stage",
             (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
             (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 21): "three_stage", (1, 1 << 22): "fused", (1, 1 << 23): "lookback",
-            (4096, 16384): "cascade_cta", (300, 65540): "cascade_cta", (160, 65540): "lookback"}
+            (4096, 16384): "cascade_cta", (300, 65540): "cascade_cta", (160, 65540): "three_stage", (120, 100003): "lookback"}
     sb.autotune_clear()
     for (G, N), algo in want.items():
         x = inputs.generate("i32", G * N, seed=G + N).reshape(G, N)
@@ -346,7 +346,8 @@ def test_auto_dispatch_regions():
     # shapes, so the choice only (both families' parity is covered above and in the fuzz)
     for (G, N), algo in {(1024, 131072): "cascade_cta", (2048, 196612): "cascade_cta",
                          (2500, 1 << 18): "cascade_cta", (2048, 1 << 18): "lookback",
-                         (1536, 196612): "lookback", (2200, 1 << 19): "lookback"}.items():
+                         (1536, 196612): "lookback", (2200, 1 << 19): "lookback",
+                         (100, 65536): "three_stage", (250, 131072): "lookback"}.items():
         xd = torch.empty((G, N), dtype=torch.int32, device="cuda")
         assert sb.plan(xd)[0] == algo, (G, N, sb.plan(xd))
         del xd

@@ -104,7 +104,7 @@ def test_paper_sweep_rates():
     x = torch.empty(T, dtype=torch.int32, device="cuda")
     inputs.fill_device(x, "i32", 5)
     y = torch.empty_like(x)
-    for n in (10, 13, 16, 20, 24, 28):
+    for n in (10, 13, 16, 17, 18, 20, 24, 28):
         N = 1 << n
         xv, yv = x.view(T // N, N), y.view(T // N, N)
         f = _frac(T, _ms(lambda: sb.scan(xv, "add", out=yv), 5))
@@ -134,3 +134,17 @@ def test_mid_size_single_problem_rates():
         xv, yv = x[:N], y[:N]
         f = _frac(N, _graph_us(lambda: sb.scan(xv, "add", out=yv)) * 1e-3)
         assert f >= FLOORS[key], (n, sb.plan(xv, yv), f)
+
+
+def test_ragged_batch_rates():
+    # problems whose starts fall inside look-back tiles, and the latency-bound middle
+    # (round 2 session 3: AUTO sends them to one CTA per problem / the three-stage form;
+    # profiles/r02_cascade_boundary.jsonl, r02_mid_batch_shapes.jsonl)
+    x = torch.empty(2048 * 65540, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 8)
+    y = torch.empty_like(x)
+    for (G, N), key in (((2048, 65540), "ragged_batch_frac_min"), ((160, 65536), "mid_batch_frac_min"),
+                        ((100, 65540), "mid_batch_frac_min")):
+        xv, yv = x[:G * N].view(G, N), y[:G * N].view(G, N)
+        f = _frac(G * N, _graph_us(lambda: sb.scan(xv, "add", out=yv)) * 1e-3)
+        assert f >= FLOORS[key], (G, N, sb.plan(xv, yv), f)
