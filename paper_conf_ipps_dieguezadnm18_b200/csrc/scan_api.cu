@@ -317,6 +317,10 @@ ChunkParams chunk_params(const void* in, void* out, int64_t N, int64_t G, scan_k
     p.in = in; p.out = out; p.N = N; p.G = G;
     p.vec = (((uintptr_t)in) % 16 == 0) && (((uintptr_t)out) % 16 == 0) && (N % 4 == 0);
     p.exclusive = kind == SCAN_EXCLUSIVE;
+    // the first wave of Stage 1 (~4 CTAs per SM) prefetches its first tiles while it waits
+    // for the previous kernel (later CTAs never wait); profiles/r02_pdl_prefetch_ab.txt
+    int sms = 0;
+    p.pf_ctas = current_device_sms(&sms) == cudaSuccess ? 4 * (int64_t)sms : 0;
     return p;
 }
 

@@ -69,6 +69,8 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_reduce_kernel(ChunkParams p)
     // stream's previous kernel -- which may trigger at entry and still be writing our
     // input -- before letting Stage 3 launch.  Otherwise Stage 1 was a normal launch and
     // everything before it is complete: trigger at once.
+    if (p.pdl_first && threadIdx.x == 0 && (int64_t)blockIdx.x < p.pf_ctas)
+        prefetch_l2_span(in + row + start, min(end - start, (int64_t)2 * TILE));
     if (p.pdl_first) grid_dep_wait();      // cross-call programmatic launch (ChunkParams)
     grid_dep_launch();          // Stage 2 / fused Stage 3 may be scheduled now
 
@@ -282,6 +284,8 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     // the next kernel on the stream may be scheduled once every CTA of this grid has
     // started (it waits for this grid's completion before touching memory)
     grid_dep_launch();
+    // (no L2 prefetch before the wait here: with it the configs[1] step lost ~1 %,
+    //  profiles/r02_pdl_prefetch_ab.txt)
     if (p.pdl_first) grid_dep_wait();      // a previous call may still be writing our input
 
     // Stage 2 results folded in: carries of earlier ranks (sharded mode),

@@ -444,6 +444,17 @@ __device__ __forceinline__ uint64_t l2_evict_last_policy() {
 __device__ __forceinline__ void prefetch_l2_bulk(const void* src, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(src), "r"(bytes) : "memory");
 }
+// Bulk L2 prefetch of the elements [p, p + n), clipped to whole 16-byte units.  Issued by
+// the cross-call programmatic kernels BEFORE their griddepcontrol.wait: a prefetch moves no
+// data to the SM and L2 is the point of coherence, so the loads after the wait still see
+// every write of the previous kernel, while the HBM -> L2 part of the first tiles overlaps
+// the previous grid's completion (~0.8 us between a CTA's entry and the end of its wait).
+template <class T>
+__device__ __forceinline__ void prefetch_l2_span(const T* p, int64_t n) {
+    if (n <= 0) return;
+    const uintptr_t a = ((uintptr_t)p + 15u) & ~(uintptr_t)15u, b = (uintptr_t)(p + n) & ~(uintptr_t)15u;
+    if (b > a) prefetch_l2_bulk((const void*)a, (uint32_t)(b - a));
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
 }

@@ -60,6 +60,7 @@ __global__ void __launch_bounds__(FU_WARPS * 32, 4) fused_grid_kernel(FusedParam
     const int64_t wb = cta * (int64_t)FU_TILE + warp * WCH;
     const T* in = (const T*)p.in;
     grid_dep_launch();
+    if (p.pdl_first && threadIdx.x == 0) prefetch_l2_span(in + cta * (int64_t)FU_TILE, min(p.total - cta * (int64_t)FU_TILE, (int64_t)FU_TILE));
     if (p.pdl_first) grid_dep_wait();            // the stream's previous kernel wrote our input
 
     // Stage 1: the tile into registers, local scan, tile aggregate

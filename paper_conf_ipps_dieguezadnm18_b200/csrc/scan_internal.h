@@ -114,6 +114,9 @@ struct ChunkParams {
     bool pdl;               // launch as a programmatic dependent of the previous kernel of
                             // this library call (Stage 2 after Stage 1, Stage 3 after Stage 2)
     PeerParams peer;        // fused exchange (peer.on) -- sharded path only
+    int64_t pf_ctas;        // Stage 1 with pdl_first: CTAs below this index (the first wave,
+                            // the ones that can start while the previous kernel drains)
+                            // L2-prefetch their first tiles before griddepcontrol.wait
 };
 int64_t chunk_tile_elems();
 int64_t warp_tile_elems();
