@@ -284,8 +284,8 @@ __global__ void __launch_bounds__(WARPS * 32) chunk_scan_kernel(ChunkParams p) {
     // the next kernel on the stream may be scheduled once every CTA of this grid has
     // started (it waits for this grid's completion before touching memory)
     grid_dep_launch();
-    // (no L2 prefetch before the wait here: with it the configs[1] step lost ~1 %,
-    //  profiles/r02_pdl_prefetch_ab.txt)
+    // (no L2 prefetch before the wait here: in large grids it cost the configs[1] step ~1 %,
+    //  in one-wave grids it was a wash: profiles/r02_pdl_prefetch_ab.txt)
     if (p.pdl_first) grid_dep_wait();      // a previous call may still be writing our input
 
     // Stage 2 results folded in: carries of earlier ranks (sharded mode),

@@ -47,6 +47,10 @@ __global__ void __launch_bounds__(WARPS * 32) cluster_scan_kernel(ChunkParams p)
     T* out = (T*)p.out + g * p.N;
     const int64_t R = (int64_t)csize * TILE;
     grid_dep_launch();                     // cross-call programmatic launch (ChunkParams)
+    // a small grid is one wave: every CTA L2-prefetches its first tile while it waits
+    // (scan_common.cuh: prefetch_l2_span)
+    if (p.pdl_first && threadIdx.x == 0 && (int64_t)gridDim.x <= p.pf_ctas)
+        prefetch_l2_span(in + (int64_t)crank * TILE, min(p.N - (int64_t)crank * TILE, (int64_t)TILE));
     if (p.pdl_first) grid_dep_wait();
 
     C run = Op::cidentity();
