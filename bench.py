@@ -589,6 +589,49 @@ def c1_latency(sb, dev, reps=50):
                     "calls; flushed = 252 MiB scratch written before each call, events around the call"}
 
 
+def g1_mid_sweep(sb, dev):
+    """One int32 problem of N = 2^22 .. 2^26 (G = 1, the paper's Fig. 11 shape),
+    where the single-GPU scan is bound by its fill and drain rather than by HBM: device time
+    per call from CUDA-graph replays of back-to-back calls, (a) "warm" on one buffer pair (as
+    the profiles/ sweeps) and (b) "cold", cycling over >= 512 MiB of distinct buffers so every
+    call reads HBM; frac = 8 B/element / time / the measured copy bandwidth, with a torch
+    copy_ of the same bytes in the same mode as the size-matched ceiling."""
+    import inputs
+    peak, _, _ = _peaks()
+    out = {}
+    gs = torch.cuda.Stream(dev)
+    for n in (22, 23, 24, 25, 26):
+        N = 1 << n
+        K = max(1, (512 << 20) // (8 * N))
+        xs = []
+        for k in range(K):
+            x = torch.empty(N, dtype=torch.int32, device=dev)
+            inputs.fill_device(x, "i32", SEED + 40 + k)
+            xs.append(x)
+        ys = [torch.empty_like(x) for x in xs]
+        reps = max(8, min(64, (1 << 30) // N * 4)) // K * K or K
+        row = {"kernel": "%s %s" % sb.plan(xs[0], ys[0])}
+        for mode, idx in (("warm", [0]), ("cold", list(range(K)))):
+            state = {"i": 0}
+
+            def call(fn_scan=True):
+                i = idx[state["i"] % len(idx)]
+                state["i"] += 1
+                if fn_scan:
+                    sb.scan(xs[i], "add", out=ys[i], stream=gs)
+                else:
+                    ys[i].copy_(xs[i])
+            r = max(reps, len(idx))
+            ms = device_time(lambda: call(True), gs, r)
+            cms = device_time(lambda: call(False), gs, r)
+            row[mode] = {"us": round(ms * 1e3, 2), "frac_measured_copy": round(8.0 * N / (ms * 1e-3) / 1e9 / peak, 4),
+                         "copy_us": round(cms * 1e3, 2), "frac_of_size_matched_copy": round(cms / ms, 4)}
+        out["2^%d" % n] = row
+        del xs, ys
+        torch.cuda.empty_cache()
+    return out
+
+
 def roofline_c3(sb, dev, budget_cpu_s: float = 10.0, reps=10, with_cpu=True):
     """configs[2]: one f32 add-scan of N = 2^30 (the L2-staged decoupled look-back), the
     north_star's ">= 80 % of HBM for N >= 2^28" point, as its own roofline line: algorithmic
@@ -904,7 +947,7 @@ def main():
         res["cpu_baseline"] = cpu_oracle_rate()
     if rank == 0 and world == 1 and not args.no_extras:
         res["roofline_c3"] = roofline_c3(sb, dev, with_cpu=not args.no_cpu)
-        res["extras"] = {"c1_i32_incl_N2^20": c1_latency(sb, dev)}
+        res["extras"] = {"c1_i32_incl_N2^20": c1_latency(sb, dev), "g1_mid_sweep": g1_mid_sweep(sb, dev)}
     if rank == 0:
         print(json.dumps(res), flush=True)
     if world > 1:

@@ -59,7 +59,8 @@ def test_c3_shape_int32_full(kind):
     (5, 3000017, "add", "i32", "inclusive"), (5, 3000017, "add", "i32", "exclusive"),
     (5, 3000017, "add", "f32s", "inclusive"), (5, 3000017, "max", "i32", "exclusive"),
     (3, 7 * 8192 * 148 + 5, "add", "u32", "inclusive"), (2048, 1 << 17, "add", "i32", "inclusive"),
-    (2048, 65540, "add", "i32", "exclusive"), (700, 200003, "add", "f32s", "inclusive")])
+    (2048, 65540, "add", "i32", "exclusive"), (700, 200003, "add", "f32s", "inclusive"),
+    (150, 200003, "max", "f32s", "exclusive"), (300, 100004, "max", "u32", "inclusive")])
 def test_lookback_multiround_segmented(G, N, op, dist, kind):
     # the persistent L2-staged look-back over MANY rounds of the CTA round robin with problem
     # starts inside tiles (segmented tiles publish P at once; the lazy look-back's window and
