@@ -68,3 +68,29 @@ def test_random_multiround_lookback(seed):
         assert_parity(to_host(out, NP[dt]).reshape(G, N), x[off:].reshape(G, N), op, kind,
                       label="fuzz-large seed=%d case=%d lookback/%d %s %s %s N=%d G=%d off=%d" % (
                           seed, case, param, op, dt, kind, N, G, off))
+
+
+@pytest.mark.parametrize("seed", range(int(__import__("os").environ.get("SCANB200_FUZZ_AUTO_SEEDS", "3"))))
+def test_random_auto_mid_batches(seed):
+    # AUTO on the batch regions re-measured in round 2 session 3 (DESIGN.md §5 items 11-12):
+    # 65 < G < 300 in the latency-bound middle (three-stage), a few hundred to a few
+    # thousand problems just above 2^16 (one CTA per problem), and their neighbours that stay
+    # on the look-back -- tile-aligned and ragged N, every op / dtype / kind
+    rng = random.Random(9000 + seed)
+    for case in range(6):
+        G = rng.choice([rng.randint(65, 299), rng.randint(300, 1100), rng.randint(1100, 3000)])
+        N = rng.choice([65536, 65540, rng.randint(65537, 140000) & ~3, rng.randint(4096, 60000) & ~3,
+                        rng.randint(140000, 300000) | 1])
+        if N * G > 40_000_000:
+            G = max(1, 40_000_000 // N)
+        op, dt = rng.choice(COMBOS)
+        kind = rng.choice(["inclusive", "exclusive"])
+        x = inputs.generate(DIST[dt], N * G, seed=seed * 100 + case + 77)
+        xd = to_device(x).view(G, N)
+        plan = sb.plan(xd, op=op, kind=kind)
+        out = sb.scan(xd, op, kind)
+        torch.cuda.synchronize()
+        assert_parity(to_host(out, NP[dt]).reshape(G, N), x.reshape(G, N), op, kind,
+                      label="fuzz-auto seed=%d case=%d %s/%d %s %s %s N=%d G=%d" % (
+                          seed, case, plan[0], plan[1], op, dt, kind, N, G))
+        del xd, out
