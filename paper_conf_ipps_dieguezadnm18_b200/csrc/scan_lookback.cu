@@ -760,8 +760,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     // the wait orders the previous kernel's writes (our input, the epoch) before any access
     grid_dep_launch();
     // the shared-memory set-up touches no global memory, so it runs before the wait for the
-    // stream's previous kernel, one ring slot per lane of warp 0 (a serial loop over the ~40
-    // barriers on one thread was ~0.7 us between CTA entry and the first bulk copy)
+    // stream's previous kernel, one ring slot per lane of warp 0 (CTA entry -> first bulk
+    // copy is ~0.8 us either way: the wait for the previous grid's completion dominates)
     static_assert(SR <= 32 && SW <= 32 && RING <= 32, "one barrier slot per lane");
     if (warp == 0) {
         if (lane < SR) { mbar_init(&fullR[lane], 1); mbar_init(&emptyR[lane], NR); }
@@ -847,8 +847,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
                     // N >= TILE: the tile holds exactly one problem start, at `first`; the
                     // chunk that contains it folds only the elements from there on (the new
                     // problem's head), every other chunk is a plain total -- a masked
-                    // reduction instead of a full segmented scan (which left seg tiles' A
-                    // ~1.7 us late and every look-back behind them re-polling)
+                    // reduction instead of a full segmented scan (ready -> A of such tiles
+                    // 2.25 -> 0.75 us, DESIGN.md §5 item 11)
                     const int first = (int)(p.N - r);
                     const int lo = k * WCH;
                     fl = first >= lo && first < lo + WCH;
