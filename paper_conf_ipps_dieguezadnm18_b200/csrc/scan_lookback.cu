@@ -367,10 +367,10 @@ __device__ __forceinline__ void tile_body_smem(const LookbackParams& p, int64_t 
 
     WarpTileS<Op, SEG, V> wt;
     {
-        const bool small = p.N < TILE;
-        int first = -1;
-        if (SEG && !small) first = r == 0 ? 0 : (int)(p.N - r);   // < TILE: SEG implies a head here
-        wt.pass1(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+        // literal `small` per call (see the L2-staged scanners): no short-problem head test
+        // in the long-problem path
+        if (SEG && p.N < TILE) wt.pass1(srow, warp * WCH, true, (uint32_t)r, (uint32_t)p.N, -1);
+        else wt.pass1(srow, warp * WCH, false, 0u, 1u, SEG ? (r == 0 ? 0 : (int)(p.N - r)) : -1);
     }
     if (lane == 0) { s_wval[warp] = wt.wtot; s_wflag[warp] = wt.wfl; }
     if (NAMED_BAR) consumer_bar(WARPS * 32); else __syncthreads();
@@ -507,10 +507,10 @@ __device__ __forceinline__ bool pipe_pass1(const LookbackParams& p, const PipeCt
     if (warp == 0 && lane == 0) trace_stamp(p, h.tid, 0);
     const T* srow = c.data + (size_t)slot * TILE + warp * WCH;
     const int64_t r = h.r;
-    if (h.seg) {
-        const bool small = p.N < TILE;
-        const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
-        st.template pass1<true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+    if (h.seg && p.N < TILE) {
+        st.template pass1<true>(srow, warp * WCH, true, (uint32_t)r, (uint32_t)p.N, -1);
+    } else if (h.seg) {
+        st.template pass1<true>(srow, warp * WCH, false, 0u, 1u, r == 0 ? 0 : (int)(p.N - r));
     } else {
         st.template pass1<false>(srow, warp * WCH, false, 0u, 1u, -1);
     }
@@ -805,11 +805,16 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const bool wpf = h.wpf[warp] != 0u, fast = h.fast != 0u;
             const int64_t gidx = t * (int64_t)TILE + warp * WCH;
             WarpTileP<Op, V> st;
-            if (h.seg) {
-                const int64_t r = h.r;
-                const bool small = p.N < TILE;
-                const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
-                st.template pass1<true>(srow, warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+            // the two head-placement modes are separate calls with a literal `small`, so each
+            // inlined copy keeps only its own head test (a runtime `small` left the per-row
+            // modulo of the short-problem test in the long-problem path: segmented tiles took
+            // 2.5 us instead of ~1 us to scan, DESIGN.md §5 item 11)
+            if (h.seg && p.N >= TILE) {
+                const int first = (int)(p.N - h.r);          // one problem start in the tile
+                st.template pass1<true>(srow, warp * WCH, false, 0u, 1u, first);
+                st.template pass2<true>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
+            } else if (h.seg) {
+                st.template pass1<true>(srow, warp * WCH, true, (uint32_t)h.r, (uint32_t)p.N, -1);
                 st.template pass2<true>(srow, (T*)p.out, gidx, p.total, fast, p.vec, p.exclusive, wp, wpf, cin);
             } else {
                 st.template pass1<false>(srow, warp * WCH, false, 0u, 1u, -1);
@@ -1095,9 +1100,8 @@ __device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t ti
     if (threadIdx.x == 0) trace_stamp(p, tile, 7);
     wt.load(in, wb, p.total, p.vec);
     if (SEG) {
-        const bool small = p.N < TILE;
-        const int first = small ? -1 : (r == 0 ? 0 : (int)(p.N - r));
-        wt.heads(warp * WCH, small, (uint32_t)(small ? r : 0), (uint32_t)(small ? p.N : 1), first);
+        if (p.N < TILE) wt.heads(warp * WCH, true, (uint32_t)r, (uint32_t)p.N, -1);
+        else wt.heads(warp * WCH, false, 0u, 1u, r == 0 ? 0 : (int)(p.N - r));
     }
     wt.scan();
     if (lane == 0) { s_wval[warp] = wt.wtot; s_wflag[warp] = wt.wfl; }
