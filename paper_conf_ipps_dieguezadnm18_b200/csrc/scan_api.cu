@@ -68,13 +68,14 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     //  tools/n12_probe.py)
     if (rows_aligned && G >= 4096 && N > 4096) return SCAN_ALGO_CASCADE_CTA;
     // hundreds to thousands of problems just above 2^16 elements, and a few thousand up to
-    // ~2^18: one CTA per problem beats the flat look-back there, by 3-74 % where problem
+    // ~2^18: one CTA per problem beats the flat look-back there, by 3-44 % where problem
     // starts fall inside look-back tiles (N not a multiple of 8192: every problem's first
     // tile needs its own look-back, the CTAs fall out of step and the round-robin
     // look-backs re-poll), ~equal on tile-aligned N (tools/cascade_boundary_probe.py,
-    // profiles/r02_cascade_boundary.jsonl); from 2^18 on at G < 2400 the look-back wins
+    // profiles/r02_cascade_boundary.jsonl, re-measured after the segmented-scan fix); from
+    // 2^18 on at G < 2400 the look-back wins; elsewhere the two are within ~3 %
     if (rows_aligned && N > 65536 &&
-        ((G >= 300 && N <= 100000) || (G >= 1024 && N <= 131072) ||
+        ((G >= 300 && N <= 81920) || (G >= 1024 && N <= 131072) ||
          (G >= 2048 && (G >= 2400 || N < 262144))))
         return SCAN_ALGO_CASCADE_CTA;
     if (rows_aligned && G >= 1184 && N >= 768 && N <= 4096) return SCAN_ALGO_CASCADE_WARP;
