@@ -16,7 +16,7 @@ import paper_conf_ipps_dieguezadnm18_b200 as sb  # noqa: E402
 from tools.paper_sweep import device_ms, peak  # noqa: E402
 
 CANDS = [("auto", -1), ("lookback", 3), ("lookback", 0), ("lookback", 1), ("lookback", 2),
-         ("cascade_cta", -1), ("three_stage", -1), ("three_stage", 1), ("three_stage", 4)]
+         ("cascade_cta", -1), ("three_stage", -1), ("three_stage", 1), ("three_stage", 4), ("fused", -1)]
 shapes = [tuple(int(v) for v in a.split("x")) for a in sys.argv[1:]]
 x = torch.empty(max(G * N for G, N in shapes), dtype=torch.int32, device="cuda")
 inputs.fill_device(x, "i32", 2018)
