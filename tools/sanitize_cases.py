@@ -46,4 +46,18 @@ for dt, dist in (("i32", "i32"), ("f32", "f32s")):
         sb.scan(x, "add", kind, algo="lookback", param=3)
         torch.cuda.synchronize()
     print("ok multi-round", dt, N, flush=True)
+# problem starts inside the L2-staged look-back's tiles (masked reduction, literal-`small`
+# head tests) and a three-stage mid batch -- the round-2 session-3 paths
+for dt, dist in (("i32", "i32"), ("f32", "f32s")):
+    for (G, N, algo, param) in ((60, 65540, "lookback", 3), (7, 3001, "lookback", 3), (70, 65536, "auto", -1)):
+        x = torch.empty(G * N, dtype=torch.int32, device="cuda")
+        inputs.fill_device(x, dist, 3)
+        if dt == "f32":
+            x = x.view(torch.float32)
+        x = x.view(G, N)
+        for kind in ("inclusive", "exclusive"):
+            sb.scan(x, "add", kind, algo=algo, param=param)
+            sb.scan(x, "max", kind, algo=algo, param=param)
+        torch.cuda.synchronize()
+        print("ok segmented", dt, G, N, algo, param, flush=True)
 print("sanitize cases done")
