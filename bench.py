@@ -376,12 +376,26 @@ def c4_problems(sb, dev, world, rank, reps=5):
             "scaling": "strong (fixed 2^32-element batch)", "kernel": kern}
 
 
+PEER_NOTE = {}
+
+
 def _peer_comms(world, max_G):
+    """The fused peer exchange (product path) and, under NCCL, the all-gather beside it.  If
+    the peer mailboxes cannot be mapped on some rank (PeerUnavailable is raised on every
+    rank alike), the legs run on the NCCL exchange alone and say so."""
     from paper_conf_ipps_dieguezadnm18_b200 import multi
-    comms = {"peer": multi.PeerComm(max_G) if world > 1 else multi.PeerComm.loopback(1, max_G)[0]}
+    comms = {}
+    try:
+        comms["peer"] = multi.PeerComm(max_G) if world > 1 else multi.PeerComm.loopback(1, max_G)[0]
+    except multi.PeerUnavailable as e:
+        PEER_NOTE["peer_unavailable"] = str(e)
     if world > 1 and DIST_BACKEND == "nccl":
         comms["nccl"] = multi.NativeComm()
     return comms
+
+
+def _product_ms(times):
+    return times["peer"] if "peer" in times else times["nccl"]
 
 
 def _time_calls(fn, reps, world):
@@ -440,6 +454,8 @@ def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB20
     # the W-rank call: fused exchange (Stage 2 pushes the totals into later ranks' HBM,
     # Stage 3 waits on the device; no collective call) is the product path, NCCL beside it
     comms = _peer_comms(world, 1)
+    if not comms:
+        return {"skipped": "no exchange available: %s" % PEER_NOTE.get("peer_unavailable", "?")}
     times = {}
     for name, c in comms.items():
         times[name] = _time_calls(lambda: multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
@@ -450,7 +466,7 @@ def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB20
         torch.distributed.barrier()
     for c in comms.values():
         c.close()
-    ms = times["peer"]
+    ms = _product_ms(times)
     # per-phase breakdown (the paper's Fig. 14): Stage 1+2 / exchange /
     # Stage 3, events between the three steps of the torch-backend path
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
@@ -483,7 +499,8 @@ def elements_mode(sb, dev, world, rank, n_local=1 << int(os.environ.get("SCANB20
             "efficiency_def": "E_W = min_r t(two-pass pipeline on the rank's portion, alone) / max_r t(W-rank "
                               "call); E_naive = min_r t(single-pass AUTO scan of the portion, alone) / max_r "
                               "t(W-rank call) (SURVEY 8(e))",
-            "exchange": ("fused peer stores in the Stage 2/3 kernels (scan_comm_create_peer)" if world > 1
+            "exchange": ("fused peer stores in the Stage 2/3 kernels (scan_comm_create_peer)" if world > 1 and "peer" in times
+                         else "NCCL all-gather (peer mailboxes unavailable)" if world > 1
                          else "none (W=1; the fused-exchange kernels run with no peers)"),
             "ms_by_exchange": times,
             "phases_ms_rank%d" % rank: {"stage1+2_reduce": ph[0], "exchange": ph[1], "stage3_scan": ph[2]}}
@@ -510,6 +527,9 @@ def scan_mps(sb, dev, world, rank, logs=(13, 20, 28), reps=10):
         x = x.view(G, L)
         y = torch.empty_like(x)
         comms = _peer_comms(world, G)
+        if not comms:
+            out["n=%d" % n] = {"skipped": "no exchange available: %s" % PEER_NOTE.get("peer_unavailable", "?")}
+            continue
         times = {}
         for name, c in comms.items():
             times[name] = _time_calls(lambda: multi.scan_multi(x, "add", "inclusive", mode="elements", out=y,
@@ -520,7 +540,7 @@ def scan_mps(sb, dev, world, rank, logs=(13, 20, 28), reps=10):
             torch.distributed.barrier()
         for c in comms.values():
             c.close()
-        ms = times["peer"]
+        ms = _product_ms(times)
         row = {"n": n, "N": N, "G": G, "N_per_gpu": L, "ms": ms, "Gelem/s": (1 << 28) / ms / 1e6,
                "per_gpu_frac_measured_hbm_at_12B": 12.0 * G * L / (ms * 1e-3) / 1e9 / hbm,
                "ms_by_exchange": times}
@@ -939,6 +959,8 @@ def main():
     torch.cuda.empty_cache()
     if not args.no_extras:
         res["elements_mode_sharded_problem"] = elements_mode(sb, dev, world, rank)
+        if PEER_NOTE:
+            res["peer_exchange_note"] = dict(PEER_NOTE)
         res["scan_mps"] = scan_mps(sb, dev, world, rank)
         res["c4_problems_mode"] = c4_problems(sb, dev, world, rank)
     if not args.no_e2e:

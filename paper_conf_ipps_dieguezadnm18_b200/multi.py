@@ -114,6 +114,10 @@ class NativeComm:
             self.handle = None
 
 
+class PeerUnavailable(RuntimeError):
+    """Raised on EVERY rank of a PeerComm set-up when any rank could not map its peers."""
+
+
 class PeerComm:
     """scan_comm_t with the fused exchange over peer memory (scan_comm_create_peer).
 
@@ -135,7 +139,21 @@ class PeerComm:
         if _open:
             blobs = [None] * self.world
             dist.all_gather_object(blobs, self.peer_handle(), group=group)
-            self.open(blobs)
+            # every rank learns whether EVERY rank mapped its peers: a rank that failed
+            # (no peer access between its GPU and another's) must not leave the others to
+            # spin on mailboxes it will never write -- all ranks raise the same error
+            err = None
+            try:
+                self.open(blobs)
+            except Exception as e:  # noqa: BLE001  (reported to every rank below)
+                err = "%s: %s" % (type(e).__name__, e)
+            errs = [None] * self.world
+            dist.all_gather_object(errs, err, group=group)
+            bad = [(r, e) for r, e in enumerate(errs) if e]
+            if bad:
+                self.close()
+                raise PeerUnavailable("peer mailboxes not mapped on rank(s) %s: %s" % (
+                    [r for r, _ in bad], bad[0][1]))
 
     def peer_handle(self) -> bytes:
         buf = ctypes.create_string_buffer(_lib.PEER_HANDLE_BYTES)

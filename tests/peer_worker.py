@@ -24,6 +24,23 @@ def main():
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     G = 3
+    if len(sys.argv) > 5 and sys.argv[5] == "failopen":
+        # rank 1 cannot map its peers: EVERY rank must get PeerUnavailable (and no rank may
+        # go on to wait on a mailbox nobody writes)
+        if rank == 1:
+            def broken_open(self, blobs):
+                raise RuntimeError("simulated: no peer access")
+            multi.PeerComm.open = broken_open
+        try:
+            multi.PeerComm(G, group=None)
+            msg = "BAD: no error"
+        except multi.PeerUnavailable as e:
+            msg = "ok-unavailable" if "simulated" in str(e) and "[1]" in str(e) else "BAD: %s" % e
+        dist.barrier()
+        with open(os.path.join(outdir, "rank%d" % rank), "w") as f:
+            f.write(msg)
+        dist.destroy_process_group()
+        return
     comm = multi.PeerComm(G, group=None)
     msg = "ok"
     try:

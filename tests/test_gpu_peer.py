@@ -135,6 +135,28 @@ def test_peer_two_processes_ipc(tmp_path):
         assert open(os.path.join(tmp_path, "rank%d" % r)).read().startswith("ok"), logs[r][-2000:]
 
 
+def test_peer_setup_failure_is_collective(tmp_path):
+    """A rank that cannot map its peers makes EVERY rank raise PeerUnavailable (bench.py then
+    runs the legs on the NCCL exchange) instead of leaving the others waiting on mailboxes."""
+    port = random.randint(20000, 40000)
+    env = dict(os.environ, PYTHONPATH=os.pathsep.join([os.path.dirname(HERE), HERE]))
+    procs = [subprocess.Popen([sys.executable, os.path.join(HERE, "peer_worker.py"), str(r), "2", str(port),
+                               str(tmp_path), "failopen"], env=env, stdout=subprocess.PIPE,
+                              stderr=subprocess.STDOUT) for r in range(2)]
+    logs = []
+    try:
+        for p in procs:
+            out, _ = p.communicate(timeout=180)
+            logs.append(out.decode(errors="replace"))
+    finally:
+        for p in procs:
+            if p.poll() is None:
+                p.kill()
+    for r, p in enumerate(procs):
+        assert p.returncode == 0, "rank %d failed:\n%s" % (r, logs[r][-3000:])
+        assert open(os.path.join(tmp_path, "rank%d" % r)).read() == "ok-unavailable", logs[r][-2000:]
+
+
 def test_c5_rank_portion_full_size():
     """configs[4] (N = 2^36 over 8 GPUs) gives every rank a 2^33-element int32 portion
     (32 GiB in + 32 GiB out).  Here the portion runs at full size as the LAST rank of a
