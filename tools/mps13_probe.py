@@ -1,0 +1,15 @@
+import os, sys
+sys.path.insert(0, "/root/repo")
+import torch, inputs
+import paper_conf_ipps_dieguezadnm18_b200 as sb
+from paper_conf_ipps_dieguezadnm18_b200 import multi
+n=13; N=1<<n; G=(1<<28)//N
+x=torch.empty(G*N,dtype=torch.int32,device="cuda"); inputs.fill_device(x,"i32",3); x=x.view(G,N); y=torch.empty_like(x)
+c=multi.PeerComm.loopback(1,G)[0]
+for _ in range(3): multi.scan_multi(x,"add","inclusive",mode="elements",out=y,backend="peer",comm=c)
+torch.cuda.synchronize()
+e0,e1=torch.cuda.Event(enable_timing=True),torch.cuda.Event(enable_timing=True)
+e0.record()
+for _ in range(10): multi.scan_multi(x,"add","inclusive",mode="elements",out=y,backend="peer",comm=c)
+e1.record(); torch.cuda.synchronize(); print("ms per call", e0.elapsed_time(e1)/10)
+c.close()
