@@ -425,16 +425,21 @@ __device__ __forceinline__ void epilogue(const LookbackParams& p, uint32_t tag) 
     if (tag + 1u >= TAG_MASK) __threadfence();
     const uint32_t prev = atomicAdd(p.ctl + 1, 1u);
     if (prev == gridDim.x - 1) {
-        __threadfence();
+        // no fences in the common case: ctl[2] was last written by the previous launch
+        // (visible across the kernel boundary) and the resets only have to be visible to
+        // the next launch, which the kernel boundary guarantees -- fences here sat on the
+        // grid's completion path (the last CTA to exit runs this)
+        if (p.epi_fence) __threadfence();
         uint32_t e = *((volatile uint32_t*)(p.ctl + 2)) + 1u;
         if (e + 1u >= TAG_MASK) {
+            __threadfence();
             for (int64_t i = 0; i < kDescWords * p.capacity; ++i) p.desc[i] = 0ull;
             e = 0u;
         }
         ((volatile uint32_t*)p.ctl)[0] = 0u;
         ((volatile uint32_t*)p.ctl)[1] = 0u;
         ((volatile uint32_t*)p.ctl)[2] = e;
-        __threadfence();
+        if (p.epi_fence || e == 0u) __threadfence();
     }
 }
 
