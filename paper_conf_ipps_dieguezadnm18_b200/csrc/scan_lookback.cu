@@ -758,6 +758,8 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     constexpr int RING = 2 * SH;             // local inclusive prefixes of this CTA's tiles
     __shared__ C s_incl[RING];
     __shared__ int64_t s_iseq[RING];
+    __shared__ uint32_t s_tag;               // the launch's descriptor tag (read once per CTA)
+    __shared__ uint64_t tagbar;              // s_tag is valid
     const int warp = threadIdx.x >> 5, lane = lane_id();
     if (threadIdx.x == 0) trace_stamp(p, blockIdx.x, 7);     // CTA entry (debug timeline)
     // every CTA is resident before a dependent grid can launch (launch_dependents counts
@@ -773,7 +775,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         if (lane < SW) { mbar_init(&fullW[lane], 1); mbar_init(&emptyW[lane], NS); }
         if (lane < SH) { mbar_init(&aggd[lane], 1); mbar_init(&crd[lane], 1); mbar_init(&emptyH[lane], NS); }
         if (lane < RING) s_iseq[lane] = -1;
-        if (lane == 0) s_end = INT64_MAX;
+        if (lane == 0) { s_end = INT64_MAX; mbar_init(&tagbar, 1); }
         fence_mbar_init();
     }
     // the HBM -> L2 part of this CTA's first SR tiles starts before that wait: a bulk L2
@@ -790,9 +792,28 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
     }
     if (p.pdl_first) grid_dep_wait();
     __syncthreads();
-    // the launch tag (an L2 round trip) is not read by the read-1 producer, so the first
-    // bulk copies are not queued behind it
-    const uint32_t tag = warp != NS + NR ? read_tag(p) : 0u;
+    // The launch tag (an L2 round trip) is read once, by the first look-back warp -- not by
+    // the read-1 producer, so the first bulk copies are not queued behind it -- and handed
+    // to the reducers and look-back warps through shared memory.  Right after reading it
+    // the CTA counts itself; the LAST CTA to have read the tag advances the epoch at once.
+    // Every CTA of this launch has then read its tag, and the next launch reads the new
+    // epoch only after this grid completed, so the advance needs no end-of-grid epilogue
+    // (an atomic round trip plus the reset on the grid's completion path).  Only a launch
+    // whose next epoch would wrap keeps the end-of-grid form (fenced, clears every slot).
+    if (warp == NS + NR + 2 && lane == 0) {
+        const uint32_t t = read_tag(p);
+        s_tag = t;
+        mbar_arrive(&tagbar);
+        if (t + 1u < TAG_MASK && atomicAdd(p.ctl + 1, 1u) == gridDim.x - 1) {
+            ((volatile uint32_t*)p.ctl)[1] = 0u;
+            ((volatile uint32_t*)p.ctl)[2] = t;        // the epoch this launch used
+        }
+    }
+    uint32_t tag = 0u;
+    if (warp >= NS && warp != NS + NR && warp != NS + NR + 1) {   // reducers, look-back warps
+        mbar_wait(&tagbar, 0u);
+        tag = s_tag;
+    }
     const T* in = (const T*)p.in;
 
     if (warp < NS) {
@@ -1019,7 +1040,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p, tag);
+    if (threadIdx.x == 0 && s_tag + 1u >= TAG_MASK) epilogue(p, s_tag);   // the wrap launch only
 }
 
 template <class Op, int NS, int NR, int SR, int SW, int SH, int M, int NLB>
