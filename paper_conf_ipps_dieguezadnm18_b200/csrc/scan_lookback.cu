@@ -449,6 +449,23 @@ __device__ __forceinline__ uint32_t read_tag(const LookbackParams& p) {
     return (e + 1u) & TAG_MASK;
 }
 
+// Start-of-grid epoch advance (see lookback_l2_kernel): a CTA counts itself right after it
+// read the launch tag (once per CTA); the ticket is consumed only at the CTA's end, so the
+// atomic's round trip overlaps the CTA's work, and the CTA that counted last advances the
+// epoch there without a further round trip.  The wrap launch keeps the fenced epilogue.
+__device__ __forceinline__ uint32_t count_tag_read(const LookbackParams& p, uint32_t tag) {
+    return tag + 1u < TAG_MASK ? atomicAdd(p.ctl + 1, 1u) : 0xFFFFFFFFu;
+}
+__device__ __forceinline__ void finish_epoch(const LookbackParams& p, uint32_t tag, uint32_t ticket) {
+    if (tag + 1u >= TAG_MASK) {
+        epilogue(p, tag);
+    } else if (ticket == gridDim.x - 1) {
+        ((volatile uint32_t*)p.ctl)[0] = 0u;
+        ((volatile uint32_t*)p.ctl)[1] = 0u;
+        ((volatile uint32_t*)p.ctl)[2] = tag;
+    }
+}
+
 
 // ---------------------------------------------------------------- pipelined, dedicated look-back warp
 // Warp roles: WARPS consumer warps, one producer warp (TMA ring), one look-back warp.
@@ -599,6 +616,8 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
         fence_mbar_init();
         s_tag = read_tag(p);
     }
+    uint32_t ticket = 0u;
+    if (threadIdx.x == 0) ticket = count_tag_read(p, s_tag);
     __syncthreads();
     const uint32_t tag = s_tag;
 
@@ -692,7 +711,7 @@ __global__ void __launch_bounds__((WARPS + 1 + NLB) * 32) lookback_pipelined_ker
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p, tag);
+    if (threadIdx.x == 0) finish_epoch(p, tag, ticket);
 }
 
 // ---------------------------------------------------------------- two reads, L2-staged (variant 3)
@@ -1090,6 +1109,8 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
         s_tile_id = tile; s_r = ti.r; s_seg = ti.seg; s_fast = ti.fast;
         s_tag = read_tag(p);
     }
+    uint32_t ticket = 0u;
+    if (threadIdx.x == 0) ticket = count_tag_read(p, s_tag);
     __syncthreads();
     const int64_t r = s_r;
     const uint32_t tag = s_tag;
@@ -1103,7 +1124,7 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
     if (s_seg) tile_body_smem<Op, true, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
     else       tile_body_smem<Op, false, WARPS, V, false>(p, tile, tag, r, s_tile, fast, &s_carry, s_wval, s_wflag);
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p, tag);
+    if (threadIdx.x == 0) finish_epoch(p, tag, ticket);
 }
 
 // ---------------------------------------------------------------- one register tile per CTA
