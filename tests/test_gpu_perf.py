@@ -125,7 +125,7 @@ def test_latency_bound_configs():
 
 def test_mid_size_single_problem_rates():
     # G = 1, N = 2^24 / 2^25 / 2^26: the L2-staged look-back's fill and drain are a large
-    # share of the call (round 2: 0.82 / 0.90 / 0.96 of copy with the lazy look-back)
+    # share of the call (round 2: 0.82-0.86 / 0.92-0.94 / 0.98 of copy after session 3)
     x = torch.empty(1 << 26, dtype=torch.int32, device="cuda")
     inputs.fill_device(x, "i32", 6)
     y = torch.empty_like(x)
