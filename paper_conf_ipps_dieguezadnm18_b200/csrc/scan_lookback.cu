@@ -1134,8 +1134,9 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_tma_kernel(LookbackParams
 // back while the others wait at one barrier; then everyone adds the carry and stores.
 // Tiles follow blockIdx (in-order dispatch, as lookback_tma_kernel).
 template <class Op, bool SEG, int WARPS, int V>
-__device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t tile, uint32_t tag, int64_t r,
-                                             typename Op::T* s_wval, uint32_t* s_wflag, typename Op::Carry* s_carry) {
+__device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t tile, uint32_t* s_tag, uint32_t& ticket,
+                                             int64_t r, typename Op::T* s_wval, uint32_t* s_wflag,
+                                             typename Op::Carry* s_carry) {
     using T = typename Op::T;
     using C = typename Op::Carry;
     constexpr int TILE = WARPS * 32 * V * 4;
@@ -1146,6 +1147,9 @@ __device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t ti
     WarpTile<Op, SEG, V> wt;
     if (threadIdx.x == 0) trace_stamp(p, tile, 7);
     wt.load(in, wb, p.total, p.vec);
+    // the launch tag is read once (thread 0, its round trip overlapping the tile's loads)
+    // and counted at once (start-of-grid epoch advance, count_tag_read)
+    if (threadIdx.x == 0) { *s_tag = read_tag(p); ticket = count_tag_read(p, *s_tag); }
     if (SEG) {
         if (p.N < TILE) wt.heads(warp * WCH, true, (uint32_t)r, (uint32_t)p.N, -1);
         else wt.heads(warp * WCH, false, 0u, 1u, r == 0 ? 0 : (int)(p.N - r));
@@ -1153,6 +1157,7 @@ __device__ __forceinline__ void regtile_body(const LookbackParams& p, int64_t ti
     wt.scan();
     if (lane == 0) { s_wval[warp] = wt.wtot; s_wflag[warp] = wt.wfl; }
     __syncthreads();
+    const uint32_t tag = *s_tag;                  // read once per CTA (thread 0), visible now
     T wp = Op::identity(); bool wpf = false;
 #pragma unroll
     for (int w = 0; w < WARPS; ++w) {
@@ -1193,13 +1198,14 @@ __global__ void __launch_bounds__(WARPS * 32) lookback_regtile_kernel(LookbackPa
     __shared__ __align__(16) T s_wval[(WARPS + 3) & ~3];   // 16-byte aligned and padded: vectorised slot reads never cover a neighbour
     __shared__ __align__(16) uint32_t s_wflag[(WARPS + 3) & ~3];
     __shared__ C s_carry;
+    __shared__ uint32_t s_tag;
     const int64_t tile = blockIdx.x;
     const TileInfo ti = classify(p, tile, TILE);
-    const uint32_t tag = read_tag(p);
-    if (ti.seg) regtile_body<Op, true, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
-    else        regtile_body<Op, false, WARPS, V>(p, tile, tag, ti.r, s_wval, s_wflag, &s_carry);
+    uint32_t ticket = 0u;
+    if (ti.seg) regtile_body<Op, true, WARPS, V>(p, tile, &s_tag, ticket, ti.r, s_wval, s_wflag, &s_carry);
+    else        regtile_body<Op, false, WARPS, V>(p, tile, &s_tag, ticket, ti.r, s_wval, s_wflag, &s_carry);
     __syncthreads();
-    if (threadIdx.x == 0) epilogue(p, tag);
+    if (threadIdx.x == 0) finish_epoch(p, s_tag, ticket);
 }
 
 // ---------------------------------------------------------------- launchers
