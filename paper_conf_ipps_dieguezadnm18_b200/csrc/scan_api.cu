@@ -257,11 +257,9 @@ const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
 // look-back options, A/B switches for on-box measurements (round 2):
 // SCANB200_LB_MODE=0 restores the round-1 speculative serialized look-back of the L2-staged
 // kernel, SCANB200_NO_KEEP_LAST=1 re-reads its last tiles, SCANB200_POLL_NS sets the first
-// back-off of a failed window poll, SCANB200_EPI_FENCE=1 restores the fences around the
-// epoch reset (the wrap launch's end-of-grid epilogue, DESIGN.md §5 item 14)
+// back-off of a failed window poll
 const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 1;
 const bool g_keep_last = std::getenv("SCANB200_NO_KEEP_LAST") == nullptr;
-const bool g_epi_fence = std::getenv("SCANB200_EPI_FENCE") != nullptr;
 const uint32_t g_poll_ns = (uint32_t)std::atoi(std::getenv("SCANB200_POLL_NS") ? std::getenv("SCANB200_POLL_NS") : "64");
 
 // debug timeline buffer for the look-back kernels (scan_debug_trace)
@@ -312,7 +310,6 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     p.lb_mode = g_lb_mode;
     p.keep_last = g_keep_last;
     p.poll_ns = g_poll_ns;
-    p.epi_fence = g_epi_fence;
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
 }
 

@@ -43,8 +43,11 @@
 //   double) written by one 128-bit store and read by one 128-bit load; a reader accepts
 //   the pair only if both tags are current and both statuses agree.  The payload is
 //   self-contained, so relaxed (.STRONG.GPU, L1-bypassing) accesses suffice.
-// The last CTA to finish resets the ticket / done counters and advances the epoch, so
-// consecutive launches (also CUDA-graph replays) need no memset.
+// Consecutive launches (also CUDA-graph replays) need no memset: every CTA reads the launch
+// tag once and counts itself at once, and the last CTA to count advances the epoch (the
+// next launch reads it only after this grid completed) -- no atomic and no fence on the
+// grid's completion path (DESIGN.md §5 item 14).  Only the launch whose next epoch would
+// wrap the 30-bit tag ends with a fenced clear of every descriptor slot.
 #include "scan_common.cuh"
 #include "scan_internal.h"
 
@@ -415,31 +418,21 @@ __device__ __forceinline__ TileInfo classify(const LookbackParams& p, int64_t t,
 }
 
 // The last CTA to finish resets the counters and advances the epoch (wrap: clear all).
-// No fence before the count in the common case: the epoch only has to advance after every
-// CTA READ it (at its start, long before); a descriptor store of this launch still in flight
-// carries this launch's tag, which no launch of the next ~2^30 accepts, so the CTA need not
-// wait for its stores here (the next kernel is ordered after this grid's completion anyway).
-// Only the launch that wraps the epoch (and clears every slot) fences first, so that none of
-// its own stores can land after the clear and survive into the next cycle of tags.
+// End-of-grid epilogue of the launch whose next epoch would wrap the 30-bit tag (tag + 1 ==
+// TAG_MASK; once per ~2^30 launches): the last CTA to finish clears every descriptor slot and
+// restarts the epoch at 0.  It fences first, so that none of this launch's own descriptor
+// stores can land after the clear and survive into the next cycle of tags.
 __device__ __forceinline__ void epilogue(const LookbackParams& p, uint32_t tag) {
-    if (tag + 1u >= TAG_MASK) __threadfence();
+    (void)tag;
+    __threadfence();
     const uint32_t prev = atomicAdd(p.ctl + 1, 1u);
     if (prev == gridDim.x - 1) {
-        // no fences in the common case: ctl[2] was last written by the previous launch
-        // (visible across the kernel boundary) and the resets only have to be visible to
-        // the next launch, which the kernel boundary guarantees -- fences here sat on the
-        // grid's completion path (the last CTA to exit runs this)
-        if (p.epi_fence) __threadfence();
-        uint32_t e = *((volatile uint32_t*)(p.ctl + 2)) + 1u;
-        if (e + 1u >= TAG_MASK) {
-            __threadfence();
-            for (int64_t i = 0; i < kDescWords * p.capacity; ++i) p.desc[i] = 0ull;
-            e = 0u;
-        }
+        __threadfence();
+        for (int64_t i = 0; i < kDescWords * p.capacity; ++i) p.desc[i] = 0ull;
         ((volatile uint32_t*)p.ctl)[0] = 0u;
         ((volatile uint32_t*)p.ctl)[1] = 0u;
-        ((volatile uint32_t*)p.ctl)[2] = e;
-        if (p.epi_fence || e == 0u) __threadfence();
+        ((volatile uint32_t*)p.ctl)[2] = 0u;
+        __threadfence();
     }
 }
 

@@ -189,19 +189,21 @@ def test_cuda_graph_replay_self_cleaning(param, N, G):
     assert_parity(to_host(out, np.float32), x, "add", "inclusive", label="graph param=%d" % param)
 
 
-def test_epoch_wrap_with_caller_workspace():
+@pytest.mark.parametrize("param", [0, 2, 3, 10])
+def test_epoch_wrap_with_caller_workspace(param):
     # poke the epoch counter of a caller workspace to just below the 30-bit wrap and run
-    # across it: the wrap path clears every descriptor
+    # across it: the wrap launch's end-of-grid epilogue clears every descriptor (every
+    # other launch advances the epoch at the start of its grid), for each look-back kernel
     N, G = 1 << 18, 3
     for op, dt in [("add", "i32"), ("add", "f32")]:
-        nbytes = sb.workspace_bytes(N, G, op, TORCH[dt], "lookback", 0)
+        nbytes = sb.workspace_bytes(N, G, op, TORCH[dt], "lookback", param)
         ws = torch.zeros((nbytes + 7) // 8, dtype=torch.int64, device="cuda")
         ctl = ws.view(torch.int32)
         ctl[2] = 0x3FFFFFFF - 4
         for it in range(8):
             x = inputs.generate(DIST[dt], N * G, 100 + it).reshape(G, N)
             xd = to_device(x)
-            out = sb.scan(xd, op, "inclusive", algo="lookback", param=0, workspace=ws)
+            out = sb.scan(xd, op, "inclusive", algo="lookback", param=param, workspace=ws)
             torch.cuda.synchronize()
             assert_parity(to_host(out, NP[dt]), x, op, "inclusive", label="wrap it=%d" % it)
         assert int(ctl[2]) < 16
