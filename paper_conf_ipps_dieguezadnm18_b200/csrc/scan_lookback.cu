@@ -417,7 +417,6 @@ __device__ __forceinline__ TileInfo classify(const LookbackParams& p, int64_t t,
     return ti;
 }
 
-// The last CTA to finish resets the counters and advances the epoch (wrap: clear all).
 // End-of-grid epilogue of the launch whose next epoch would wrap the 30-bit tag (tag + 1 ==
 // TAG_MASK; once per ~2^30 launches): the last CTA to finish clears every descriptor slot and
 // restarts the epoch at 0.  It fences first, so that none of this launch's own descriptor
