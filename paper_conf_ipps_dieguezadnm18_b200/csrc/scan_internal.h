@@ -38,7 +38,8 @@ struct LookbackParams {
     void* out;
     int64_t N;          // elements per problem (> 0)
     int64_t total;      // G * N
-    uint32_t* ctl;      // [0] ticket, [1] done, [2] epoch   (zero-initialised once)
+    uint32_t* ctl;      // [0] (unused, kept 0), [1] CTAs that read this launch's tag,
+                        // [2] epoch   (zero-initialised once)
     uint64_t* desc;     // descriptors: value<<32|tag<<2|status (two such words per tile for fp64)
     int64_t capacity;   // 16-byte descriptor slots of the workspace (>= tiles of any call)
     uint64_t* trace;    // debug: 4 %globaltimer stamps per tile (NULL in normal use)
