@@ -1,5 +1,8 @@
+"""Scan-MPS at W = 1, n = 13 (G = 32768 problems of 8192): the elements-mode call with the
+fused-exchange communicator of one rank, ms per call from events around 10 calls (for an
+ncu launch list of the pipeline's kernels)."""
 import os, sys
-sys.path.insert(0, "/root/repo")
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch, inputs
 import paper_conf_ipps_dieguezadnm18_b200 as sb
 from paper_conf_ipps_dieguezadnm18_b200 import multi
