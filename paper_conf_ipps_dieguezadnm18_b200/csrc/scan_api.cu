@@ -260,6 +260,11 @@ const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
 // back-off of a failed window poll
 const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 1;
 const bool g_keep_last = std::getenv("SCANB200_NO_KEEP_LAST") == nullptr;
+// the L2-staged kernel's read 2 at the tile's aggregate instead of its carry: 3-7 % faster
+// up to 2^28 elements, a wash (+-2 %) above (profiles/r02_lb_early_read2_ab.txt);
+// SCANB200_EARLY_READ2=1 / SCANB200_LATE_READ2=1 force either form at every size (A/B)
+const bool g_early_read2_all = std::getenv("SCANB200_EARLY_READ2") != nullptr;
+const bool g_late_read2_all = std::getenv("SCANB200_LATE_READ2") != nullptr;
 const uint32_t g_poll_ns = (uint32_t)std::atoi(std::getenv("SCANB200_POLL_NS") ? std::getenv("SCANB200_POLL_NS") : "64");
 
 // debug timeline buffer for the look-back kernels (scan_debug_trace)
@@ -310,6 +315,7 @@ scan_status run_lookback(const void* in, void* out, int64_t N, int64_t G, scan_o
     p.lb_mode = g_lb_mode;
     p.keep_last = g_keep_last;
     p.poll_ns = g_poll_ns;
+    p.early_read2 = !g_late_read2_all && (g_early_read2_all || total <= (int64_t(1) << 28));
     return from_cuda(launch_lookback(opcode(op, dt), p, variant, s));
 }
 

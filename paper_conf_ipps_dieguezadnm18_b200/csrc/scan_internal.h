@@ -54,6 +54,7 @@ struct LookbackParams {
     bool keep_last;     // L2-staged kernel: each CTA's last tile is scanned from the read-1
                         // ring slot (no second read on the kernel's critical tail)
     uint32_t poll_ns;   // first back-off of a failed look-back poll (look_back_par / _rr)
+    bool early_read2;   // L2-staged kernel: read 2 at the tile's aggregate, not its carry
 };
 // u64 words per look-back descriptor slot.  A descriptor needs 1 (32-bit carries) or 2
 // (fp64 carries) words; one descriptor per 64-byte slot puts only two tiles on a 128-byte

@@ -835,6 +835,7 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
             const SlotHdr<Op, NS>& h = s_hdr[sH];
             const int64_t t = h.tid;
             if (t < 0) break;
+            if (p.early_read2) mbar_wait(&crd[sH], (uint32_t)((i / SH) & 1));   // the carry
             // a kept tile (the CTA's last) is still in its read-1 slot: no second read
             const T* srow = (h.keep ? bufR + (size_t)(i % SR) * TILE : bufW + (size_t)sW * TILE) + warp * WCH;
             const T cin = Op::from_carry(h.carry);
@@ -973,7 +974,11 @@ __global__ void __launch_bounds__((NS + NR + 2 + NLB) * 32, 1) lookback_l2_kerne
         const uint64_t pol = l2_evict_first_policy();
         for (int64_t i = 0;; ++i) {
             const int sW = (int)(i % SW), sH = (int)(i % SH);
-            mbar_wait(&crd[sH], (uint32_t)((i / SH) & 1));
+            // read 2 goes out once the tile's carry is known -- or, with early_read2, once
+            // its aggregate is (the data waits in the W ring instead of in L2 while the
+            // look-back resolves; the scanners then wait for the carry themselves)
+            if (p.early_read2) mbar_wait(&aggd[sH], (uint32_t)((i / SH) & 1));
+            else mbar_wait(&crd[sH], (uint32_t)((i / SH) & 1));
             mbar_wait(&emptyW[sW], (uint32_t)((i / SW) & 1) ^ 1u);
             const SlotHdr<Op, NS>& h = s_hdr[sH];
             const int64_t t = h.tid;
