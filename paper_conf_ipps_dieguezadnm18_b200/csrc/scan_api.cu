@@ -99,13 +99,14 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // 13.2 us against 12.5 / 12.5 us i32 / f32; 7 x 2^20: 15.5 against 14.2 / 15.0 us;
     // profiles/r02_fused_probe_tpc2_REVERTED.jsonl)
     if (G <= 64 && N * G <= (int64_t(1) << 22) && N >= 4096) return SCAN_ALGO_THREE_STAGE;
-    // tens to a few hundred problems of up to ~2^17 elements, 2^22 < G*N <= 2^24: the
-    // latency-bound middle, where the three-stage form (its second read still hits L2)
-    // beats both the look-back and one CTA per problem (e.g. G = 160, N = 65536: 0.74 vs
-    // 0.70 / 0.54 of copy; G = 100, N = 65540: 0.60 vs 0.43; tools/shape_probe.py,
-    // profiles/r02_mid_batch_shapes.jsonl)
-    if (rows_aligned && G > 64 && G < 300 && N >= 4096 && N <= 131076 && N * G > (int64_t(1) << 22) &&
-        N * G <= (int64_t(1) << 24))
+    // tens to a few hundred problems of up to ~80K elements, 2^22 < G*N <= 2^24, problem
+    // starts inside look-back tiles: the latency-bound middle, where the three-stage form
+    // (its second read still hits L2) beats both the look-back and one CTA per problem
+    // (G = 100, N = 65540: 0.59 vs 0.53 / 0.43 of copy; G = 160, N = 32772: 0.54 vs 0.43 /
+    // 0.44).  Tile-aligned or longer rows stay on the look-back since its session-3 changes
+    // (G = 200, N = 65536: 0.83 vs 0.71; tools/shape_probe.py, profiles/r02_mid_batch_shapes.jsonl)
+    if (rows_aligned && G > 64 && G < 300 && N >= 4096 && N <= 81920 && N % 8192 != 0 &&
+        N * G > (int64_t(1) << 22) && N * G <= (int64_t(1) << 24))
         return SCAN_ALGO_THREE_STAGE;
     // a few hundred to a few thousand problems of moderate length (scan_autotune over a
     // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA

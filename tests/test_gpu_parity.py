@@ -349,7 +349,7 @@ def test_auto_dispatch_regions():
     for (G, N), algo in {(1024, 131072): "cascade_cta", (2048, 196612): "cascade_cta",
                          (2500, 1 << 18): "cascade_cta", (2048, 1 << 18): "lookback",
                          (1536, 196612): "lookback", (2200, 1 << 19): "lookback",
-                         (100, 65536): "three_stage", (250, 131072): "lookback"}.items():
+                         (100, 65536): "lookback", (100, 65540): "three_stage", (250, 131072): "lookback"}.items():
         xd = torch.empty((G, N), dtype=torch.int32, device="cuda")
         assert sb.plan(xd)[0] == algo, (G, N, sb.plan(xd))
         del xd
