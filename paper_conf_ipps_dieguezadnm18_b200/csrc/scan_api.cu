@@ -261,6 +261,8 @@ const bool g_cross_pdl = std::getenv("SCANB200_NO_PDL") == nullptr;
 // back-off of a failed window poll
 const int g_lb_mode = std::getenv("SCANB200_LB_MODE") ? std::atoi(std::getenv("SCANB200_LB_MODE")) : 1;
 const bool g_keep_last = std::getenv("SCANB200_NO_KEEP_LAST") == nullptr;
+// sharded path: warp-per-problem Stage 1 / Stage 3 for short portions (SCANB200_NO_WARP_SHARD=1: A/B)
+const bool g_warp_shard = std::getenv("SCANB200_NO_WARP_SHARD") == nullptr;
 // the L2-staged kernel's read 2 at the tile's aggregate instead of its carry: 3-7 % faster
 // up to 2^28 elements, a wash (+-2 %) above (profiles/r02_lb_early_read2_ab.txt);
 // SCANB200_EARLY_READ2=1 / SCANB200_LATE_READ2=1 force either form at every size (A/B)
@@ -360,8 +362,12 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
         p.pdl = true;                                        // Stage 3 overlaps Stage 1's tail
         return from_cuda(launch_chunk_scan(oc, p, s));
     }
+    // many short portions (one chunk per problem): Stage 1 and Stage 3 with one warp per
+    // problem (profiles/r02_mps_phases_W1.jsonl: one CTA per problem idled at N <= 2048)
+    const bool warp_path = p.Bx == 1 && N <= 4096 && G >= 1184 && g_warp_shard;
     if (stages12) {
-        cudaError_t e = launch_chunk_reduce(oc, p, s);       // normal launch: waits for the caller's work
+        cudaError_t e = warp_path ? launch_warp_reduce(oc, p, s)    // normal launch: waits for
+                                  : launch_chunk_reduce(oc, p, s);  // the caller's work
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
         p.pdl = true;                                        // Stage 2 overlaps Stage 1's tail
         e = launch_aux_scan(oc, p, s);
@@ -370,7 +376,7 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
     // Stage 3 directly after this library's Stage 2 (same call, or the fused-exchange
     // path) starts early and loads its first tile while Stage 2 finishes
     p.pdl = stages12 || pdl3;
-    if (stage3) return from_cuda(launch_chunk_scan(oc, p, s));
+    if (stage3) return from_cuda(warp_path ? launch_warp_shard_scan(oc, p, s) : launch_chunk_scan(oc, p, s));
     return SCAN_OK;
 }
 

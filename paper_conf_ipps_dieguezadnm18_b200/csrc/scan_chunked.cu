@@ -401,6 +401,87 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
     }
 }
 
+// ------------------------------------------------------------------ warp per problem, sharded path
+// Short portions (N_local <= 4096, one chunk per problem, many problems): Stage 1 and
+// Stage 3 of the sharded pipeline with one WARP per problem
+// instead of one 256-thread CTA per (problem, chunk), which left most of each CTA idle
+// (N_local = 1024: Stage 1 0.33, Stage 3 0.28 of copy; profiles/r02_mps_phases_W1.jsonl).
+// Stage 1: the raw reduction of the warp's problem into aux[g * Bx] (Bx == 1).
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) warp_reduce_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    if (p.pdl_first) grid_dep_wait();      // the library's ordering rule (chunk_reduce_kernel)
+    grid_dep_launch();
+    if (g >= p.G) return;
+    const int64_t row = g * p.N;
+    const T* in = (const T*)p.in;
+    C acc = Op::cidentity();
+    for (int64_t off = 0; off < p.N; off += WCH) {
+        Row4<T> x[V];
+#pragma unroll
+        for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, row + off + j * 128 + lane * 4, row + p.N, p.vec);
+        T t = Op::identity();
+#pragma unroll
+        for (int j = 0; j < V; ++j)
+#pragma unroll
+            for (int k = 0; k < 4; ++k) t = Op::apply(t, x[j].v[k]);
+        acc = Op::capply(acc, Op::to_carry(t));
+    }
+    acc = warp_reduce_carry<Op>(acc);
+    if (lane == 0) p.aux[g * p.Bx] = slot_put(acc);
+}
+
+// Stage 3: carry = the totals of the ranks before this one (fused exchange: wait for their
+// rows in this rank's mailbox, then acknowledge once every CTA has read -- as
+// chunk_scan_kernel's fold_carry), then the warp cascade over the problem.  With one chunk
+// per problem the chunk prefix of Stage 2 is the identity.  Launched as a dependent of
+// Stage 2: waits for it before any access.
+template <class Op, int WARPS, int V>
+__global__ void __launch_bounds__(WARPS * 32) warp_shard_scan_kernel(ChunkParams p) {
+    using T = typename Op::T;
+    using C = typename Op::Carry;
+    constexpr int WCH = V * 128;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    const bool live = g < p.G;
+    grid_dep_launch();
+    grid_dep_wait();
+    C carry = Op::cidentity();
+    const int64_t stride = p.carry_stride ? p.carry_stride : p.G;
+    const bool peer_wait = p.peer.on && p.peer.rank > 0;
+    if (peer_wait) {
+        if (live && lane == 0) {
+            for (int r = 0; r < p.peer.rank; ++r) peer_wait_ge(p.peer.my_flags + r, p.peer.epoch);
+            for (int r = 0; r < p.carry_rows; ++r)
+                carry = Op::capply(carry, slot_get<C>(ld_relaxed_sys_u64(p.carry_src + (int64_t)r * stride + g)));
+        }
+        carry = shfl_idx_c<C>(carry, 0);
+    } else if (live) {
+        for (int r = 0; r < p.carry_rows; ++r) carry = Op::capply(carry, slot_get<C>(p.carry_src[(int64_t)r * stride + g]));
+    }
+    if (live) {
+        const int64_t row = g * p.N;
+        const T* in = (const T*)p.in;
+        T* out = (T*)p.out;
+        for (int64_t off = 0; off < p.N; off += WCH) {
+            WarpTile<Op, false, V> wt;
+            wt.load(in, row + off, row + p.N, p.vec);
+            wt.scan();
+            wt.store(out, row + off, row + p.N, p.vec, Op::identity(), false, Op::from_carry(carry), p.exclusive);
+            carry = Op::capply(carry, Op::to_carry(wt.wtot));
+        }
+    }
+    if (peer_wait) {
+        __syncthreads();                   // every warp of the CTA has read its mailbox row
+        if (threadIdx.x == 0 && peer_last_cta(p.peer.counters + 1))
+            for (int r = 0; r < p.peer.rank; ++r) st_release_sys_u64(p.peer.push_ack[r], p.peer.epoch);
+    }
+}
+
 // ------------------------------------------------------------------ packed short problems
 // Several whole problems per warp (L_x < 32 threads per problem): warp w owns
 // problems [w*k, (w+1)*k) -- one contiguous span of k*N elements that starts and ends on
@@ -575,6 +656,20 @@ cudaError_t warp_op(const ChunkParams& p, cudaStream_t s) {
     return launch_maybe_pdl(warp_cascade_kernel<Op, WC_WARPS, WC_V>, (unsigned)blocks, WC_WARPS * 32, p, s);
 }
 template <class Op>
+cudaError_t warp_reduce_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = (p.G + WC_WARPS - 1) / WC_WARPS;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    if (blocks == 0) return cudaSuccess;
+    return launch_maybe_pdl(warp_reduce_kernel<Op, WC_WARPS, WC_V>, (unsigned)blocks, WC_WARPS * 32, p, s);
+}
+template <class Op>
+cudaError_t warp_shard_scan_op(const ChunkParams& p, cudaStream_t s) {
+    int64_t blocks = (p.G + WC_WARPS - 1) / WC_WARPS;
+    if (blocks > 0x7FFFFFFF) return cudaErrorInvalidConfiguration;
+    if (blocks == 0) return cudaSuccess;
+    return launch_maybe_pdl(warp_shard_scan_kernel<Op, WC_WARPS, WC_V>, (unsigned)blocks, WC_WARPS * 32, p, s);
+}
+template <class Op>
 cudaError_t packed_op(const ChunkParams& p, cudaStream_t s) {
     const bool pow2 = p.N > 0 && p.N <= 512 && (p.N & (p.N - 1)) == 0;
     if (pow2 && p.vec) {                                   // regular segments, one window per warp
@@ -613,6 +708,8 @@ cudaError_t launch_chunk_reduce(OpCode op, const ChunkParams& p, cudaStream_t s)
 cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(auxscan_op) }
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(scan_op) }
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_op) }
+cudaError_t launch_warp_reduce(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_reduce_op) }
+cudaError_t launch_warp_shard_scan(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(warp_shard_scan_op) }
 cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s) { SCANB200_DISPATCH(packed_op) }
 cudaError_t launch_peer_ack(const PeerParams& pp, cudaStream_t s) {
     if (!pp.on || pp.rank == 0) return cudaSuccess;

@@ -132,6 +132,9 @@ cudaError_t launch_aux_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 cudaError_t launch_chunk_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 // Warp-per-problem cascade (L_y = warps per block problems per CTA).
 cudaError_t launch_warp_cascade(OpCode op, const ChunkParams& p, cudaStream_t s);
+// sharded path with short portions (Bx == 1): Stage 1 / Stage 3 with one warp per problem
+cudaError_t launch_warp_reduce(OpCode op, const ChunkParams& p, cudaStream_t s);
+cudaError_t launch_warp_shard_scan(OpCode op, const ChunkParams& p, cudaStream_t s);
 // Packed short problems: p.chunk = k whole problems per warp span (k*N % 4 == 0 when
 // p.vec), segmented scan, no carry between spans (L_x < 32).
 cudaError_t launch_packed_warp(OpCode op, const ChunkParams& p, cudaStream_t s);

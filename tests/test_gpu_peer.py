@@ -66,6 +66,46 @@ def test_peer_loopback_parity(W):
             c.close()
 
 
+@pytest.mark.parametrize("W", [2, 4])
+def test_short_portions_warp_path(W):
+    # many problems with short per-rank portions (N_local <= 4096, G >= 1184) take the
+    # warp-per-problem Stage 1 / Stage 3 (scan_api.cu run_three_stage); ranks with longer
+    # or empty portions take the CTA path / the bare acknowledgement in the same call, so
+    # the mixed paths must interoperate through the mailboxes.  Both exchanges: the fused
+    # peer stores and the public two-step API with the totals stacked on the host side.
+    rng = random.Random(17 + W)
+    for op, dt in COMBOS:
+        G = rng.choice([1184, 1500, 3000])
+        lens = [rng.choice([0, 1, 37, 1000, 2048, 4096, 4097, 6000]) for _ in range(W)]
+        if sum(lens) == 0:
+            lens[0] = 100
+        Ntot = sum(lens)
+        x = inputs.generate(DIST[dt], G * Ntot, seed=W * 1000 + len(op) + Ntot).reshape(G, Ntot)
+        starts = np.cumsum([0] + lens)
+        parts = [to_device(np.ascontiguousarray(x[:, starts[r]:starts[r] + L])) for r, L in enumerate(lens)]
+        comms = multi.PeerComm.loopback(W, G)
+        try:
+            for kind in ("inclusive", "exclusive"):
+                outs = _run_loopback(comms, parts, op, kind)
+                torch.cuda.synchronize()
+                got = np.concatenate([to_host(o, NP[dt]).reshape(G, -1) for o in outs], axis=1)
+                assert_parity(got, x, op, kind, label="warp-path peer W=%d %s %s %s G=%d lens=%s" % (
+                    W, op, dt, kind, G, lens))
+        finally:
+            torch.cuda.synchronize()
+            for c in comms:
+                c.close()
+        # the public steps: Stage 1+2 on every rank, the [W, G] totals stacked, Stage 3
+        for kind in ("inclusive", "exclusive"):
+            tots = [sb.shard_totals(xl, op) for xl in parts]
+            allt = torch.stack(tots)
+            outs = [sb.shard_scan(xl, allt, r, W, op, kind) for r, xl in enumerate(parts)]
+            torch.cuda.synchronize()
+            got = np.concatenate([to_host(o, NP[dt]).reshape(G, -1) for o in outs], axis=1)
+            assert_parity(got, x, op, kind, label="warp-path steps W=%d %s %s %s G=%d lens=%s" % (
+                W, op, dt, kind, G, lens))
+
+
 def test_peer_loopback_many_epochs_graph_free():
     # 64 back-to-back calls with no host sync in between: the ack protocol alone keeps
     # a mailbox half from being overwritten before the later ranks read it

@@ -1,6 +1,7 @@
 """Soak test of the fused peer-memory exchange (scan_comm_create_peer) with W real ranks
 (W processes sharing cuda:0, CUDA-IPC-mapped mailboxes, gloo plumbing): many consecutive
-elements-mode calls with random G and random (uneven, sometimes empty) portions -- the
+elements-mode calls with random G (up to 2048: the short-portion
+warp path too) and random (uneven, sometimes empty) portions -- the
 mailbox halves, flags and acknowledgements cycle through hundreds of epochs.  Every 7th
 call is checked against the oracle of the whole batch.
 
@@ -29,12 +30,15 @@ def rank_main(rank, world, iters, port):
     os.environ["MASTER_PORT"] = str(port)
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    comm = multi.PeerComm(64)
+    comm = multi.PeerComm(2048)
     rng = random.Random(1234)                   # identical sequence on every rank
     bad = 0
     for it in range(iters):
-        G = rng.choice([1, 1, 2, 3, 17, 64])
-        lens = [rng.choice([0, 1, 5, 4096, 9000, 70001]) for _ in range(world)]
+        G = rng.choice([1, 1, 2, 3, 17, 64, 1300, 2048])
+        if G > 64:      # many short portions: the warp-per-problem Stage 1 / Stage 3 (N_local <= 4096)
+            lens = [rng.choice([0, 1, 37, 1000, 2048, 4096, 5000]) for _ in range(world)]
+        else:
+            lens = [rng.choice([0, 1, 5, 4096, 9000, 70001]) for _ in range(world)]
         if sum(lens) == 0:
             lens[-1] = 3
         Ntot = sum(lens)
