@@ -363,11 +363,14 @@ scan_status run_three_stage(const void* in, void* out, int64_t N, int64_t G, sca
         return from_cuda(launch_chunk_scan(oc, p, s));
     }
     // many short portions (one chunk per problem): Stage 1 and Stage 3 with one warp per
-    // problem (profiles/r02_mps_phases_W1.jsonl: one CTA per problem idled at N <= 2048)
+    // problem (profiles/r02_mps_phases_W1.jsonl: one CTA per problem idled at N <= 2048);
+    // Stage 2 is folded into Stage 1 there (one chunk per problem: only the totals move)
     const bool warp_path = p.Bx == 1 && N <= 4096 && G >= 1184 && g_warp_shard;
-    if (stages12) {
-        cudaError_t e = warp_path ? launch_warp_reduce(oc, p, s)    // normal launch: waits for
-                                  : launch_chunk_reduce(oc, p, s);  // the caller's work
+    if (stages12 && warp_path) {
+        // Stages 1+2 in one launch (the warp stores and pushes its problem's total)
+        if (launch_warp_reduce(oc, p, s) != cudaSuccess) return SCAN_ERR_CUDA;
+    } else if (stages12) {
+        cudaError_t e = launch_chunk_reduce(oc, p, s);       // normal launch: waits for the caller's work
         if (e != cudaSuccess) return SCAN_ERR_CUDA;
         p.pdl = true;                                        // Stage 2 overlaps Stage 1's tail
         e = launch_aux_scan(oc, p, s);

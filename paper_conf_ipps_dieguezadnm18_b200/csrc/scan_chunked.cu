@@ -406,7 +406,11 @@ __global__ void __launch_bounds__(WARPS * 32) warp_cascade_kernel(ChunkParams p)
 // Stage 3 of the sharded pipeline with one WARP per problem
 // instead of one 256-thread CTA per (problem, chunk), which left most of each CTA idle
 // (N_local = 1024: Stage 1 0.33, Stage 3 0.28 of copy; profiles/r02_mps_phases_W1.jsonl).
-// Stage 1: the raw reduction of the warp's problem into aux[g * Bx] (Bx == 1).
+// Stages 1+2 in one kernel: with one chunk per problem Stage 2 is the identity on the chunk
+// prefixes and only copies each problem's total out (and pushes it to the later ranks'
+// mailboxes) -- a separate aux_scan launch of G/8 CTAs cost 60 us at G = 2^18 for 2 MB, so
+// the warp stores its total directly with aux_scan_kernel's exchange protocol (wait for the
+// acks of call epoch-2 before overwriting a mailbox half; the last CTA raises the flags).
 template <class Op, int WARPS, int V>
 __global__ void __launch_bounds__(WARPS * 32) warp_reduce_kernel(ChunkParams p) {
     using T = typename Op::T;
@@ -414,25 +418,44 @@ __global__ void __launch_bounds__(WARPS * 32) warp_reduce_kernel(ChunkParams p) 
     constexpr int WCH = V * 128;
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const int64_t g = (int64_t)blockIdx.x * WARPS + warp;
+    const bool live = g < p.G;
+    const PeerParams& pp = p.peer;
+    const bool push = pp.on && pp.rank + 1 < pp.ngpu;      // someone reads this rank's totals
     if (p.pdl_first) grid_dep_wait();      // the library's ordering rule (chunk_reduce_kernel)
     grid_dep_launch();
-    if (g >= p.G) return;
-    const int64_t row = g * p.N;
-    const T* in = (const T*)p.in;
     C acc = Op::cidentity();
-    for (int64_t off = 0; off < p.N; off += WCH) {
-        Row4<T> x[V];
+    if (live) {
+        const int64_t row = g * p.N;
+        const T* in = (const T*)p.in;
+        for (int64_t off = 0; off < p.N; off += WCH) {
+            Row4<T> x[V];
 #pragma unroll
-        for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, row + off + j * 128 + lane * 4, row + p.N, p.vec);
-        T t = Op::identity();
+            for (int j = 0; j < V; ++j) x[j] = load_row<Op>(in, row + off + j * 128 + lane * 4, row + p.N, p.vec);
+            T t = Op::identity();
 #pragma unroll
-        for (int j = 0; j < V; ++j)
+            for (int j = 0; j < V; ++j)
 #pragma unroll
-            for (int k = 0; k < 4; ++k) t = Op::apply(t, x[j].v[k]);
-        acc = Op::capply(acc, Op::to_carry(t));
+                for (int k = 0; k < 4; ++k) t = Op::apply(t, x[j].v[k]);
+            acc = Op::capply(acc, Op::to_carry(t));
+        }
+        acc = warp_reduce_carry<Op>(acc);
     }
-    acc = warp_reduce_carry<Op>(acc);
-    if (lane == 0) p.aux[g * p.Bx] = slot_put(acc);
+    if (push) {
+        // the mailbox half this call writes was last read by call epoch-2 of ranks > rank
+        if (threadIdx.x == 0 && pp.epoch > 2)
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) peer_wait_ge(pp.my_acks + q, pp.epoch - 2);
+        __syncthreads();
+    }
+    if (live && lane == 0) {
+        p.totals[g] = slot_put(acc);
+        if (push)
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) st_relaxed_sys_u64(pp.push_totals[q] + g, slot_put(acc));
+    }
+    if (push) {
+        __syncthreads();
+        if (threadIdx.x == 0 && peer_last_cta(pp.counters + 0))
+            for (int q = pp.rank + 1; q < pp.ngpu; ++q) st_release_sys_u64(pp.push_flag[q], pp.epoch);
+    }
 }
 
 // Stage 3: carry = the totals of the ranks before this one (fused exchange: wait for their
