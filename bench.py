@@ -399,9 +399,16 @@ def _product_ms(times):
 
 
 def _time_calls(fn, reps, world):
-    """Device time per call (events on the launching stream), max over ranks."""
-    for _ in range(3):
+    """Device time per call (events on the launching stream), max over ranks.  Warm-up of at
+    least 10 calls AND 50 ms: with three calls, the first point of a leg (Scan-MPS n = 13)
+    read 0.585 ms instead of 0.47 ms, with ten 0.535 ms -- a time-based ramp after the idle
+    host work before the leg, which later points and standalone runs never showed."""
+    t0, calls = time.perf_counter(), 0
+    while calls < 10 or time.perf_counter() - t0 < 0.05:
         fn()
+        calls += 1
+        if calls % 10 == 0:
+            torch.cuda.synchronize()
     torch.cuda.synchronize()
     align_ranks(world)
     s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
