@@ -84,6 +84,9 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // (~2.5-3.3 us per call against 5-12 us for three-stage / look-back), one thread-block
     // cluster per problem (DSMEM aggregates) up to 2^15: ~3.3-3.9 us
     if (G <= 148 && N <= 8192) return SCAN_ALGO_CASCADE_CTA;
+    // ... and for 64 < G <= 148 up to ~20K elements (G = 80-140, N = 9220-16388: 0.18-0.33 of
+    // copy against 0.10-0.21 for the look-back; profiles/r02_mid_batch_dispatch.jsonl)
+    if (rows_aligned && G > 64 && G <= 148 && N > 8192 && N < 20480) return SCAN_ALGO_CASCADE_CTA;
     // (2^15 < N <= 2^16 at G = 1: the two-launch chain 3.6 us vs the cluster 3.9-4.0 us once
     //  both use programmatic launch, profiles/r01_g1_probe_cluster_boundary.jsonl)
     if (G <= 64 && N <= 32768) return SCAN_ALGO_CLUSTER;
@@ -108,6 +111,16 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     if (rows_aligned && G > 64 && G < 300 && N >= 4096 && N <= 81920 && N % 8192 != 0 &&
         N * G > (int64_t(1) << 22) && N * G <= (int64_t(1) << 24))
         return SCAN_ALGO_THREE_STAGE;
+    // the same below 2^22 elements for 64 < G <= 148, tile-aligned or not (G = 70 / 100 / 128,
+    // N = 20484-40964: 0.25-0.47 of copy against 0.18-0.42 for the look-back; 100 x 32768:
+    // 0.50 vs 0.36; profiles/r02_mid_batch_dispatch.jsonl)
+    if (rows_aligned && G > 64 && G <= 148 && N >= 20480 && N * G <= (int64_t(1) << 22))
+        return SCAN_ALGO_THREE_STAGE;
+    // tile-aligned rows of 40960-65536 elements, 148 < G <= 600: the look-back (every problem
+    // starts on a tile) beats one CTA per problem (G = 200, N = 65536: 0.81 vs 0.63; G = 500:
+    // 0.92 vs 0.79); from G = 800 the cascade wins again (profiles/r02_mid_batch_dispatch.jsonl)
+    if (rows_aligned && G > 148 && G <= 600 && N >= 40960 && N <= 65536 && N % 8192 == 0)
+        return SCAN_ALGO_LOOKBACK;
     // a few hundred to a few thousand problems of moderate length (scan_autotune over a
     // G x N grid, profiles/r01_autotune_probe.jsonl): whole problems per warp / per CTA
     // beat the flat look-back 1.1-4.8x there (e.g. G = 1024, N = 4096: 5.9 us vs 28 us)

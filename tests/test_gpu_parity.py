@@ -335,7 +335,8 @@ def test_auto_dispatch_regions():
     want = {(1, 4096): "cascade_cta", (100, 8192): "cascade_cta", (1, 20000): "cluster", (4, 32768): "cluster", (4, 65536): "three_stage",
             (64, 65536): "three_stage", (1, 1 << 20): "three_stage", (1000, 1000): "cascade_warp",
             (256, 4096): "cascade_cta", (1024, 65536): "cascade_cta", (1, 1 << 21): "three_stage", (1, 1 << 22): "fused", (1, 1 << 23): "lookback",
-            (4096, 16384): "cascade_cta", (300, 65540): "cascade_cta", (160, 65540): "three_stage", (120, 100003): "lookback"}
+            (4096, 16384): "cascade_cta", (300, 65540): "cascade_cta", (160, 65540): "three_stage", (120, 100003): "lookback",
+            (100, 20484): "three_stage", (160, 40960): "lookback", (100, 12292): "cascade_cta"}
     sb.autotune_clear()
     for (G, N), algo in want.items():
         x = inputs.generate("i32", G * N, seed=G + N).reshape(G, N)
@@ -349,7 +350,11 @@ def test_auto_dispatch_regions():
     for (G, N), algo in {(1024, 131072): "cascade_cta", (2048, 196612): "cascade_cta",
                          (2500, 1 << 18): "cascade_cta", (2048, 1 << 18): "lookback",
                          (1536, 196612): "lookback", (2200, 1 << 19): "lookback",
-                         (100, 65536): "lookback", (100, 65540): "three_stage", (250, 131072): "lookback"}.items():
+                         (100, 65536): "lookback", (100, 65540): "three_stage", (250, 131072): "lookback",
+                         # profiles/r02_mid_batch_dispatch.jsonl
+                         (200, 65536): "lookback", (500, 49152): "lookback", (800, 65536): "cascade_cta",
+                         (200, 65532): "three_stage", (100, 32772): "three_stage", (70, 20484): "three_stage",
+                         (100, 32768): "three_stage", (140, 10244): "cascade_cta"}.items():
         xd = torch.empty((G, N), dtype=torch.int32, device="cuda")
         assert sb.plan(xd)[0] == algo, (G, N, sb.plan(xd))
         del xd

@@ -17,6 +17,11 @@ from tools.paper_sweep import device_ms, peak  # noqa: E402
 
 CANDS = [("auto", -1), ("lookback", 3), ("lookback", 0), ("lookback", 1), ("lookback", 2),
          ("cascade_cta", -1), ("three_stage", -1), ("three_stage", 1), ("three_stage", 4), ("fused", -1)]
+if os.environ.get("SHAPE_PROBE_MID"):          # the mid-batch dispatch boundary
+    CANDS = [("auto", -1), ("lookback", 3), ("lookback", 1), ("cascade_cta", -1), ("three_stage", -1)]
+if os.environ.get("SHAPE_PROBE_CLUSTER"):      # the cluster family: param = 32 * variant + csize
+    CANDS = [("auto", -1), ("three_stage", -1), ("lookback", 3)] + [
+        ("cluster", 32 * v + c) for v in (0, 1, 2) for c in (4, 8, 16)]
 shapes = [tuple(int(v) for v in a.split("x")) for a in sys.argv[1:]]
 x = torch.empty(max(G * N for G, N in shapes), dtype=torch.int32, device="cuda")
 inputs.fill_device(x, "i32", 2018)
