@@ -87,6 +87,9 @@ scan_algo choose_algo(int64_t N, int64_t G, bool aligned) {
     // ... and for 64 < G <= 148 up to ~20K elements (G = 80-140, N = 9220-16388: 0.18-0.33 of
     // copy against 0.10-0.21 for the look-back; profiles/r02_mid_batch_dispatch.jsonl)
     if (rows_aligned && G > 64 && G <= 148 && N > 8192 && N < 20480) return SCAN_ALGO_CASCADE_CTA;
+    // G just under the SM count: one CTA per problem is one full wave (G = 148, N = 20484-32772:
+    // 0.53-0.62 of copy against 0.42-0.53 three-stage; G = 140: a tie)
+    if (rows_aligned && G > 140 && G <= 148 && N > 8192 && N < 36864) return SCAN_ALGO_CASCADE_CTA;
     // (2^15 < N <= 2^16 at G = 1: the two-launch chain 3.6 us vs the cluster 3.9-4.0 us once
     //  both use programmatic launch, profiles/r01_g1_probe_cluster_boundary.jsonl)
     if (G <= 64 && N <= 32768) return SCAN_ALGO_CLUSTER;

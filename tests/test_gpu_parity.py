@@ -354,7 +354,8 @@ def test_auto_dispatch_regions():
                          # profiles/r02_mid_batch_dispatch.jsonl
                          (200, 65536): "lookback", (500, 49152): "lookback", (800, 65536): "cascade_cta",
                          (200, 65532): "three_stage", (100, 32772): "three_stage", (70, 20484): "three_stage",
-                         (100, 32768): "three_stage", (140, 10244): "cascade_cta"}.items():
+                         (100, 32768): "three_stage", (140, 10244): "cascade_cta", (148, 28676): "cascade_cta",
+                         (132, 28676): "three_stage"}.items():
         xd = torch.empty((G, N), dtype=torch.int32, device="cuda")
         assert sb.plan(xd)[0] == algo, (G, N, sb.plan(xd))
         del xd
