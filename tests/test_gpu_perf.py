@@ -148,3 +148,37 @@ def test_ragged_batch_rates():
         xv, yv = x[:G * N].view(G, N), y[:G * N].view(G, N)
         f = _frac(G * N, _graph_us(lambda: sb.scan(xv, "add", out=yv)) * 1e-3)
         assert f >= FLOORS[key], (G, N, sb.plan(xv, yv), f)
+
+
+def test_short_portion_sharded_rates():
+    # the sharded pipeline with short per-rank portions (warp per problem, DESIGN §8 item 4):
+    # Scan-MPS at W = 8 for n <= 15 gives each rank G >= 8192 portions of <= 4096 elements.
+    # Stage 1+2 reads 4 B/elem, Stage 3 moves 8 B/elem (profiles/r02_warp_shard_ab.txt:
+    # 1.13 / 1.02 of copy at N_local = 1024; the CTA path read 0.33 / 0.28)
+    T = 1 << 28
+    x = torch.empty(T, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 9)
+    y = torch.empty_like(x)
+    for N in (1024, 4096):
+        G = T // N
+        xv, yv = x.view(G, N), y.view(G, N)
+        tot = sb.shard_totals(xv, "add")
+        allt = tot.view(1, G).clone()
+        us12 = _graph_us(lambda: sb.shard_totals(xv, "add", totals=tot))
+        us3 = _graph_us(lambda: sb.shard_scan(xv, allt, 0, 1, "add", "inclusive", out=yv))
+        f12 = _frac(T, us12 * 1e-3) / 2          # 4 B/elem
+        f3 = _frac(T, us3 * 1e-3)
+        assert f12 >= FLOORS["short_portion_stage12_frac_min"], (N, f12)
+        assert f3 >= FLOORS["short_portion_stage3_frac_min"], (N, f3)
+
+
+def test_mid_batch_aligned_rates():
+    # tile-aligned rows of 40960-65536 elements at 148 < G <= 600 (look-back since the
+    # 60-shape grid, profiles/r02_mid_batch_dispatch_final.jsonl: 0.68-0.93 of copy)
+    x = torch.empty(600 * 65536, dtype=torch.int32, device="cuda")
+    inputs.fill_device(x, "i32", 10)
+    y = torch.empty_like(x)
+    for G, N in ((200, 65536), (500, 49152), (600, 65536)):
+        xv, yv = x[:G * N].view(G, N), y[:G * N].view(G, N)
+        f = _frac(G * N, _graph_us(lambda: sb.scan(xv, "add", out=yv)) * 1e-3)
+        assert f >= FLOORS["mid_aligned_frac_min"], (G, N, sb.plan(xv, yv), f)
